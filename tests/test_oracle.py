@@ -1,0 +1,327 @@
+"""Oracle pins (CPU only).  Each test pins an oracle function to something other than
+itself: published test vectors, a published inverse, brute force on tiny inputs, closed
+forms, and invariants the paper states.  See DESIGN.md §4 for the pin table."""
+import json
+import os
+import random
+import struct
+
+import numpy as np
+import pytest
+
+import oracle
+import wdgen
+
+GOLD = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "hash_vectors.json")))
+
+
+# ------------------------------------------------------------------ (1) hash functions
+def murmur3_x86_32(data: bytes, seed: int) -> int:
+    """MurmurHash3_x86_32 body (SMHasher); its finalisation step is the ORACLE's fmix32,
+    so the published vectors pin fmix32."""
+    c1, c2, M = 0xCC9E2D51, 0x1B873593, 0xFFFFFFFF
+    rotl = lambda x, r: ((x << r) | (x >> (32 - r))) & M
+    h = seed & M
+    nblocks = len(data) // 4
+    for i in range(nblocks):
+        (k,) = struct.unpack_from("<I", data, 4 * i)
+        k = (k * c1) & M; k = rotl(k, 15); k = (k * c2) & M
+        h ^= k; h = rotl(h, 13); h = (h * 5 + 0xE6546B64) & M
+    tail = data[4 * nblocks:]
+    k = 0
+    if len(tail) >= 3: k ^= tail[2] << 16
+    if len(tail) >= 2: k ^= tail[1] << 8
+    if len(tail) >= 1:
+        k ^= tail[0]; k = (k * c1) & M; k = rotl(k, 15); k = (k * c2) & M; h ^= k
+    h ^= len(data)
+    return oracle.fmix32(h)
+
+
+@pytest.mark.parametrize("vec", GOLD["murmur3_x86_32"])
+def test_fmix32_published_murmur3_vectors(vec):
+    assert murmur3_x86_32(bytes.fromhex(vec["data_hex"]), vec["seed"]) == int(vec["hash"], 16)
+
+
+def _mueller_inverse(y: np.ndarray) -> np.ndarray:
+    """Mueller's published inverse (tests/golden/hash_vectors.json)."""
+    x = y.astype(np.uint64)
+    inv = np.uint64(int(GOLD["mueller_inverse_multiplier"], 16))
+    m = np.uint64(0xFFFFFFFF)
+    x = (((x >> np.uint64(16)) ^ x) * inv) & m
+    x = (((x >> np.uint64(16)) ^ x) * inv) & m
+    x = (x >> np.uint64(16)) ^ x
+    return x.astype(np.uint32)
+
+
+def _fmix32_inverse(y: np.ndarray) -> np.ndarray:
+    """Inverse of the MurmurHash3 finalizer (inverses of xorshift and of the odd
+    multipliers 0x85ebca6b^-1 = 0xa5cb9243, 0xc2b2ae35^-1 = 0x7ed1b41d)."""
+    m = np.uint64(0xFFFFFFFF)
+    x = y.astype(np.uint64)
+    x ^= x >> np.uint64(16)
+    x = (x * np.uint64(0x7ED1B41D)) & m
+    x ^= (x >> np.uint64(13)) ^ (x >> np.uint64(26))
+    x = (x * np.uint64(0xA5CB9243)) & m
+    x ^= x >> np.uint64(16)
+    return x.astype(np.uint32)
+
+
+def test_inverse_multipliers():
+    assert (0x45D9F3B * 0x119DE1F3) & 0xFFFFFFFF == 1
+    assert (0x85EBCA6B * 0xA5CB9243) & 0xFFFFFFFF == 1
+    assert (0xC2B2AE35 * 0x7ED1B41D) & 0xFFFFFFFF == 1
+
+
+def test_hashes_are_bijections_p161():
+    # both functions "act as isomorphism on the space of 4-byte integers".
+    # A left inverse on every tested point proves injectivity there; 2^22 random points
+    # plus the edges.
+    rng = np.random.default_rng(0)
+    x = np.concatenate([rng.integers(0, 2**32, 1 << 22, dtype=np.uint64).astype(np.uint32),
+                        np.array([0, 1, 2, 0x7FFFFFFF, 0x80000000, 0xFFFFFFFE, 0xFFFFFFFF],
+                                 np.uint32)])
+    assert np.array_equal(_mueller_inverse(oracle.mueller_many(x)), x)
+    assert np.array_equal(_fmix32_inverse(oracle.fmix32_many(x)), x)
+    assert oracle.fmix32(0) == 0 and oracle.mueller(0) == 0
+
+
+# ------------------------------------------------------------------ (2) partition
+def test_partition_range_and_balance():
+    keys = wdgen.unique_keys(1 << 20, seed=1)
+    for m in (1, 2, 3, 4, 8):
+        d = oracle.partition(keys, m, seed=0x9E3779B9)
+        assert d.max() < m
+        cnt = np.bincount(d, minlength=m)
+        mu = keys.size / m
+        assert np.all(np.abs(cnt - mu) < 6 * np.sqrt(mu) + 1)
+
+
+def test_partition_fig4_mode():
+    keys = np.arange(28, dtype=np.uint32) * 7 + 3
+    assert np.array_equal(oracle.partition(keys, 4, 0, oracle.PART_MOD), keys % 4)
+
+
+def test_partition_decorrelated_from_table_hash():
+    # C15: keys of one partition must spread over the whole table hash range
+    keys = wdgen.unique_keys(1 << 16, seed=2)
+    d = oracle.partition(keys, 8, seed=0x9E3779B9)
+    h = oracle.fmix32_many(keys[d == 3]) >> np.uint32(29)  # top 3 bits of the table hash
+    cnt = np.bincount(h, minlength=8)
+    assert cnt.min() > 0.8 * cnt.mean()
+
+
+# ------------------------------------------------------------------ (3) the map
+def _brute_map(calls):
+    """Pure-Python dictionary over a list of insert calls (C8)."""
+    d, pairs, lastcall, paircall = {}, set(), {}, {}
+    for ci, (ks, vs) in enumerate(calls):
+        for k, v in zip(ks, vs):
+            k, v = int(k), int(v)
+            if k == 0xFFFFFFFF:
+                continue
+            d[k] = v
+            pairs.add((k, v)); lastcall[k] = ci; paircall[(k, v)] = ci
+    return d, pairs, lastcall, paircall
+
+
+@pytest.mark.parametrize("trial", range(20))
+def test_map_matches_bruteforce_tiny(trial):
+    rnd = random.Random(trial)
+    domain = [rnd.randrange(0, 2**32) for _ in range(40)] + [0, 0xFFFFFFFF, 0xFFFFFFFE]
+    calls = []
+    for _ in range(rnd.randint(1, 4)):
+        n = rnd.randint(0, 64)
+        ks = [rnd.choice(domain) for _ in range(n)]
+        vs = [rnd.choice([0, 1, 0xFFFFFFFF, rnd.randrange(2**32)]) for _ in range(n)]
+        calls.append((ks, vs))
+    m = oracle.Map(4, dup_mode=True)  # tiny initial capacity: exercises growth
+    skipped = 0
+    for ks, vs in calls:
+        skipped += m.insert(np.array(ks, np.uint32), np.array(vs, np.uint32))
+    d, pairs, lastcall, paircall = _brute_map(calls)
+    assert m.size() == len(d)
+    assert skipped == sum(int(k) == 0xFFFFFFFF for ks, _ in calls for k in ks)
+    q = np.array(domain + [rnd.randrange(2**32) for _ in range(20)], np.uint32)
+    vals, found = m.retrieve(q)
+    for k, v, f in zip(q, vals, found):
+        k = int(k)
+        if k in d:
+            assert f == 1 and int(v) == d[k]
+        else:
+            assert f == 0 and int(v) == 0xFFFFFFFF
+    # pair-set membership (duplicate mode)
+    for (k, v) in list(pairs)[:50]:
+        st = int(m.pair_status(np.array([k], np.uint32), np.array([v], np.uint32))[0])
+        assert st == (2 if paircall[(k, v)] == lastcall[k] else 1)
+    assert int(m.pair_status(np.array([5], np.uint32), np.array([12345], np.uint32))[0]) in (0, 1, 2)
+
+
+def test_map_closed_form_unique_mode():
+    n, ks, vs = 1 << 16, 21, 22
+    keys, vals = wdgen.unique_keys(n, ks), wdgen.values(n, vs)
+    m = oracle.Map(n)
+    assert m.insert(keys, vals) == 0
+    assert m.size() == n
+    q = wdgen.interleaved_queries(n, ks)
+    gv, gf = m.retrieve(q)
+    ev, ef = oracle.expected_unique(q, n, ks, vs)
+    assert np.array_equal(gf, ef) and np.array_equal(gv, ev)
+    assert gf.sum() == n  # half present, half absent
+
+
+def test_map_load_is_size_over_capacity():
+    # P:63 alpha = n / c for unique keys; the north-star invariant load = size/capacity
+    n = 5000
+    m = oracle.Map(n)
+    m.insert(wdgen.unique_keys(n, 1), wdgen.values(n, 1))
+    m.insert(wdgen.unique_keys(n // 2, 1), wdgen.values(n // 2, 2))  # updates only
+    assert m.size() == n
+
+
+# ------------------------------------------------------------------ (4) multisplit
+def test_multisplit_bruteforce():
+    rng = np.random.default_rng(3)
+    for m in (1, 2, 3, 4, 8):
+        keys = rng.integers(0, 2**32, 777, dtype=np.uint64).astype(np.uint32)
+        counts, perm = oracle.multisplit(keys, m, seed=99)
+        d = oracle.partition(keys, m, 99)
+        # brute force: stable sort by destination
+        order = sorted(range(keys.size), key=lambda i: (int(d[i]), i))
+        want_perm = np.empty(keys.size, np.uint64)
+        want_perm[order] = np.arange(keys.size)
+        assert np.array_equal(perm, want_perm)
+        assert np.array_equal(counts, np.bincount(d, minlength=m).astype(np.uint64))
+
+
+def test_multisplit_fig4_shape():
+    # Fig. 4: 4 GPUs x 7 keys, p(k) = k mod 4.  The paper's concrete keys are only
+    # in the image, so we use our own 28 keys with the same partition function.
+    keys = np.array([5, 12, 7, 0, 3, 3, 9, 14, 2, 1, 8, 11, 6, 4, 13, 10, 15, 0, 7, 2, 9,
+                     21, 18, 16, 27, 22, 25, 19], np.uint32)
+    out = []
+    for g in range(4):
+        kg = keys[7 * g:7 * g + 7]
+        counts, perm = oracle.multisplit(kg, 4, 0, oracle.PART_MOD)
+        res = np.empty(7, np.uint32)
+        res[perm.astype(np.int64)] = kg
+        # each partition is contiguous, holds exactly keys = d (mod 4), in input order
+        off = 0
+        for dd in range(4):
+            part = res[off:off + int(counts[dd])]
+            assert np.all(part % 4 == dd)
+            assert list(part) == [k for k in kg if k % 4 == dd]
+            off += int(counts[dd])
+        out.append(counts)
+    T = np.array(out, np.uint64)
+    assert T.sum() == 28
+    assert np.array_equal(T.sum(axis=0), np.bincount(keys % 4, minlength=4))
+
+
+# ------------------------------------------------------------------ (5) T scans
+def test_table_scans_bruteforce():
+    rng = np.random.default_rng(4)
+    for m in (1, 2, 4, 8):
+        T = rng.integers(0, 1000, (m, m)).astype(np.uint64)
+        so, ro = oracle.table_scans(T)
+        for g in range(m):
+            for p in range(m):
+                assert so[g, p] == T[g, :p].sum()
+                assert ro[p, g] == T[:g, p].sum()
+        # transposition isomorphism: every (g,p) block lands in a disjoint range on p
+        for p in range(m):
+            ends = ro[p] + T[:, p]
+            assert ends[-1] == T[:, p].sum()
+            assert np.all(ro[p][1:] == ends[:-1])
+
+
+# ------------------------------------------------------------------ (6) Fig. 3 replay
+@pytest.mark.parametrize("G", [1, 2, 4, 8, 16, 32])
+def test_replay_single_region_closed_form(G):
+    # c = 32: one region, every p maps to base 0, so Fig. 3 scans slots 0..31 left to
+    # right: the i-th distinct key lands in slot i after i//G + 1 windows, touching
+    # ceil((i//G + 1) * G / 4) sectors; the 33rd key exhausts p_max regions (Line 26).
+    pmax = 3
+    r = oracle.Replay(32, G, p_max=pmax)
+    keys = wdgen.unique_keys(33, seed=5)
+    vals = wdgen.values(33, seed=5)
+    for i in range(32):
+        w0, s0 = r.ins.windows, r.ins.sectors
+        r.insert(keys[i:i + 1], vals[i:i + 1])
+        assert r.ins.windows - w0 == i // G + 1
+        assert r.ins.sectors - s0 == -(-((i // G + 1) * G) // 4)
+        assert int(r.table[i]) == (int(vals[i]) << 32) | int(keys[i])
+    assert r.ins.new_keys == 32 and r.ins.failures == 0
+    w0 = r.ins.windows
+    r.insert(keys[32:], vals[32:])
+    assert r.ins.failures == 1 and r.ins.windows - w0 == pmax * (32 // G)
+    # full table: a query for an absent key also exhausts p_max (C10)
+    v, f = r.query(keys[32:])
+    assert f[0] == 0 and v[0] == 0xFFFFFFFF and r.qry.windows == pmax * (32 // G)
+    v, f = r.query(keys[:32])
+    assert np.all(f == 1) and np.array_equal(v, vals[:32])
+
+
+def test_replay_base_range():
+    for c in (32, 36, 100, 1000, 1103768, 2**33 + 4):
+        for k in (0, 1, 0xDEADBEEF, 0xFFFFFFFE):
+            for p in range(0, 50, 7):
+                b = oracle.Replay.base(k, p, c)
+                assert 0 <= b <= c - 32 and b % 4 == 0
+    # bases over many keys cover the whole range [0, c-32] roughly uniformly
+    c = 4096
+    bs = np.array([oracle.Replay.base(int(k), 0, c) for k in wdgen.unique_keys(20000, 1)])
+    hist = np.bincount(bs // 4, minlength=(c - 32) // 4 + 1)
+    assert hist.min() >= 1 and hist.max() < 5 * hist.mean()
+
+
+def test_replay_layout_independent_of_group_size_p89():
+    # "The inner probing loop (Line 6) ensures a consistent probing scheme in case
+    # that the size of g is varied": the sequential layout must not depend on |g|.
+    n, c = 6000, 6320
+    keys = wdgen.unique_keys(n, 8)
+    vals = wdgen.values(n, 8)
+    tables = []
+    for G in (1, 2, 4, 8, 16, 32):
+        r = oracle.Replay(c, G)
+        r.insert(keys, vals)
+        assert r.ins.new_keys == n
+        tables.append(r.table.copy())
+    for t in tables[1:]:
+        assert np.array_equal(t, tables[0])
+
+
+@pytest.mark.parametrize("dup", [False, True])
+def test_replay_results_equal_map(dup):
+    # the replay of Fig. 3 reaches the same map as the plain dictionary (sequential
+    # upserts, last value wins), for hits, misses and updates
+    n = 20000
+    c = (int(n / 0.95) + 3) // 4 * 4
+    if dup:
+        keys = wdgen.uniform_keys(n, 3) % np.uint32(9000)  # many repeats
+    else:
+        keys = wdgen.unique_keys(n, 3)
+    vals = wdgen.values(n, 4)
+    r = oracle.Replay(c, 4)
+    r.insert(keys, vals)
+    m = oracle.Map(n)
+    m.insert(keys, vals)
+    assert r.ins.new_keys == m.size() and r.ins.failures == 0
+    q = np.concatenate([keys, wdgen.unique_keys(5000, 3, start=n)])
+    rv, rf = r.query(q)
+    mv, mf = m.retrieve(q)
+    assert np.array_equal(rf, mf) and np.array_equal(rv, mv)
+
+
+def test_replay_probe_costs_grow_with_load():
+    # sanity of the cost model: windows/op increase with alpha, decrease with |g|
+    n = 1 << 15
+    keys, vals = wdgen.unique_keys(n, 1), wdgen.values(n, 1)
+    w = {}
+    for a in (0.8, 0.95):
+        c = (int(n / a) + 3) // 4 * 4
+        for G in (1, 4, 32):
+            r = oracle.Replay(c, G)
+            r.insert(keys, vals)
+            w[a, G] = r.ins.windows / n
+    assert w[0.8, 4] < w[0.95, 4]
+    assert w[0.95, 1] > w[0.95, 4] > w[0.95, 32] >= 1.0
