@@ -1,0 +1,410 @@
+#!/usr/bin/env python
+"""bench.py — WarpDrive hot path on B200: G inserts/s + G queries/s at load 0.95.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--sweep]
+
+One step = one pass of the whole hot path over one batch of synthetic input
+(SURVEY §8(a)): a1 table fill, a2+a3 insert of n unique pairs, a2+a4 retrieve of the same
+n keys (100 % hits; BASELINE config 2's "insert and retrieve" at alpha = 0.95, |g| = 4);
+with N > 1 (torchrun, one process per GPU, weak scaling: n pairs per GPU) the insert and
+retrieve run the distributed cascades a6-a10 (multisplit fused with the NVLink push, T
+flags, local probe, reverse pull + unpermute).
+
+value      = (inserts + queries of all ranks) / max-over-ranks step time, device-resident
+             inputs, CUDA events on the launching stream.
+e2e        = the same step through the C-ABI with PINNED HOST buffers: H2D of keys/values/
+             queries and D2H of values/found inside the timed region (out-of-core path a11).
+roofline   = the dominant kernel (per-launch CUDA-event time inside the timed region)
+             against the measured HBM copy bandwidth (MEASURED_PEAKS.json), with the
+             ALGORITHMIC bytes of SURVEY §8(d): insert 8 + 32 S_ins + 32 B, hit query
+             9 + 32 S_hit B, S from the oracle's sequential Fig. 3 replay
+             (tests/golden/probe_cost.json, written by tools/probe_cost.py).
+cpu_baseline = the oracle (single-threaded C dictionary) on a bounded sample.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "G inserts/s and G queries/s at load 0.95, 1/2/4/8 B200; % HBM sector roofline"
+UNIT = "G ops/s"
+KEY_SEED, VAL_SEED = 0x5EED, 0xBEEF
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n-log2", type=int, default=28, help="pairs per GPU (config 2: 28)")
+    ap.add_argument("--alpha", type=float, default=0.95)
+    ap.add_argument("--group-size", type=int, default=4)
+    ap.add_argument("--kif", type=int, default=0, help="keys in flight per group (0=default)")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--sweep", action="store_true",
+                    help="extra lines: config-2 alpha x |g| sweep (not the headline)")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index, self.rows, self.proc = index, [], None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        sm = [float(r[0]) for r in self.rows if len(r) >= 7 and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) >= 7 and r[1].replace(".", "").isdigit()]
+        reasons = sorted({names[i] for r in self.rows if len(r) >= 7
+                          for i in range(4) if r[3 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- helpers
+def probe_cost(alpha: float, G: int):
+    d = json.load(open(os.path.join(ROOT, "tests", "golden", "probe_cost.json")))
+    best = min(d["rows"], key=lambda r: (abs(r["alpha"] - alpha), abs(r["G"] - G)))
+    return best
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def cpu_baseline_sample(log2n: int = 24):
+    """The oracle as it stands (single-threaded C dictionary), on a bounded sample of the
+    same workload: 2^log2n unique inserts + 2^log2n hit queries."""
+    import numpy as np
+    import oracle
+    import wdgen
+    n = 1 << log2n
+    keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
+    m = oracle.Map(n)
+    t0 = time.perf_counter()
+    m.insert(keys, vals)
+    t1 = time.perf_counter()
+    v, f = m.retrieve(keys)
+    t2 = time.perf_counter()
+    assert int(f.sum()) == n and np.array_equal(v, vals)
+    return {"value": 2 * n / (t2 - t0) / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"2^{log2n} unique inserts + 2^{log2n} hit queries (config-2 workload, "
+                      f"bounded), single-threaded C dictionary",
+            "insert_gops": n / (t1 - t0) / 1e9, "query_gops": n / (t2 - t1) / 1e9,
+            "seconds": t2 - t0, "host_cpus": os.cpu_count()}
+
+
+# ----------------------------------------------------------------------------- reference arm
+def run_reference(args):
+    """--impl reference: the oracle (this tier's reference arm) on the host cores, on the
+    same config/metric; each step a bounded sample (2^22 inserts + 2^22 queries)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import numpy as np
+    import oracle
+    import wdgen
+    n = 1 << 22
+    keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
+    times = []
+    for it in range(args.warmup + args.steps):
+        m = oracle.Map(n)
+        t0 = time.perf_counter()
+        m.insert(keys, vals)
+        v, f = m.retrieve(keys)
+        dt = time.perf_counter() - t0
+        m.close()
+        if it >= args.warmup:
+            times.append(dt)
+    t = sum(times) / len(times)
+    val = 2 * n / t / 1e9
+    line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic", "impl": "reference",
+            "config": {"workload": "config2: 2^28 unique u32 pairs, alpha 0.95, |g| 4, "
+                                   "insert + retrieve (reference arm: bounded 2^22 sample per step)",
+                       "global_batch": n, "alpha": args.alpha, "group_size": args.group_size},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": "2^22 unique inserts + 2^22 hit queries per step"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- our arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_junger0s18_b200 as wd
+    import wdgen.gpu as gg
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    assert world == args.gpus or world == 1, "launch N>1 with torchrun --nproc-per-node N"
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+
+    n = 1 << args.n_log2
+    G = args.group_size
+    cap_local = int(math.ceil(n / args.alpha))
+    if world > 1:
+        uid = wd.Table.unique_id() if rank == 0 else None
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        table = wd.Table(cap_local * world, group_size=G, rank=rank, world=world,
+                         unique_id=obj[0])
+    else:
+        table = wd.Table(cap_local, 1, G)
+    if args.kif:
+        table.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, args.kif)
+
+    # inputs: rank r inserts generator indices [r n, (r+1) n) -> globally unique keys
+    keys = gg.unique_keys(n, KEY_SEED, start=rank * n)
+    vals = gg.values(n, VAL_SEED, start=rank * n)
+    vout = torch.empty(n, dtype=torch.int32, device="cuda")
+    fout = torch.empty(n, dtype=torch.uint8, device="cuda")
+    stream = torch.cuda.current_stream()
+    torch.cuda.synchronize()
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+
+    def step(marks=None):
+        table.clear(stream)
+        if marks is not None:
+            marks[0].record(stream)
+        table.insert(keys, vals, stream)
+        if marks is not None:
+            marks[1].record(stream)
+        table.retrieve(keys, vout, fout, stream)
+        if marks is not None:
+            marks[2].record(stream)
+
+    # ---- warm-up + correctness of the measured configuration (sampled, closed form)
+    for _ in range(args.warmup):
+        step()
+    barrier()
+    st = table.sync()
+    assert st == 0, f"device-side status {st}: {wd._lib.wd_last_error_message()}"
+    assert table.size() == n * world
+    idx = torch.randint(0, n, (1 << 16,), device="cuda")
+    ok = bool((fout[idx] == 1).all().item()) and bool((vout[idx] == vals[idx]).all().item())
+    assert ok, "measured configuration returned wrong results"
+
+    # ---- timed region: device-resident
+    launches0 = table.launches
+    marks = [[ev(), ev(), ev()] for _ in range(args.steps)]
+    e0, e1 = ev(), ev()
+    with ClockSampler(local_rank) as clk:
+        barrier()
+        e0.record(stream)
+        for k in range(args.steps):
+            step(marks[k])
+        e1.record(stream)
+        barrier()
+    launches = table.launches - launches0
+    t_ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+    ins_ms = max_over_ranks(sum(a.elapsed_time(b) for a, b, _ in marks) / args.steps)
+    qry_ms = max_over_ranks(sum(b.elapsed_time(c) for _, b, c in marks) / args.steps)
+    ops = 2 * n * world
+    value = ops / (t_ms * 1e-3) / 1e9
+    assert table.sync() == 0
+
+    # ---- roofline of the dominant kernel (single GPU: one launch per call)
+    pc = probe_cost(args.alpha, G)
+    hbm, peak_src = peaks()
+    b_ins = 8 + 32 * pc["ins_sectors"] + 32
+    b_hit = 9 + 32 * pc["hit_sectors"]
+    kern = {"insert": (ins_ms, b_ins), "retrieve": (qry_ms, b_hit)}
+    dom = max(kern, key=lambda k: kern[k][0])
+    other = "retrieve" if dom == "insert" else "insert"
+
+    def roof(name):
+        ms, bpo = kern[name]
+        ach = n * bpo / (ms * 1e-3) / 1e9
+        return {"kernel": f"probe_kernel<{name}> (G={G})", "bound": "hbm", "achieved": ach,
+                "peak": hbm, "unit": "GB/s", "frac": ach / hbm, "traffic": None,
+                "bytes_per_op": bpo, "launch_ms": ms,
+                "sectors_per_op": pc["ins_sectors" if name == "insert" else "hit_sectors"]}
+
+    roofline = roof(dom)
+    roofline["peak_source"] = peak_src
+    roofline["other"] = roof(other)
+    traffic_file = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(traffic_file) and world == 1:
+        tr = json.load(open(traffic_file)).get(f"{dom}_G{G}_a{args.alpha}_n{args.n_log2}")
+        if tr:
+            roofline["traffic"] = tr
+
+    # ---- e2e: the same step through the C-ABI with pinned host buffers
+    e2e = None
+    if not args.no_e2e:
+        hk = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        hv = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        hk.copy_(keys)
+        hv.copy_(vals)
+        hvo = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        hfo = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        table.set_option(wd.WD_OPT_BATCH, 1 << 24)
+
+        def hstep():
+            table.clear(stream)
+            table.insert(hk, hv, stream)
+            table.retrieve(hk, hvo, hfo, stream)
+
+        hstep()
+        barrier()
+        assert bool((hfo[:4096] == 1).all()) and bool((hvo[:4096] == hv[:4096]).all())
+        e_steps = max(1, min(args.steps, 5))
+        a, b = ev(), ev()
+        barrier()
+        a.record(stream)
+        for _ in range(e_steps):
+            hstep()
+        b.record(stream)
+        barrier()
+        te = max_over_ranks(a.elapsed_time(b) / e_steps)
+        e2e = {"value": ops / (te * 1e-3) / 1e9, "unit": UNIT, "ms_per_step": te,
+               "h2d_bytes_per_step": 12 * n, "d2h_bytes_per_step": 5 * n, "steps": e_steps}
+        assert table.sync() == 0
+
+    # ---- CPU baseline (rank 0, N = 1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline_sample(24)
+
+    sweep_lines = []
+    if args.sweep and world == 1:
+        sweep_lines = run_sweep(args, wd, gg, torch)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_ms,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"config2: 2^{args.n_log2} unique u32 key/value pairs per GPU, "
+                                   f"load {args.alpha}, |g|={G}; step = fill + insert all + "
+                                   f"retrieve all (100% hits)",
+                       "global_batch": n * world, "pairs_per_gpu": n, "alpha": args.alpha,
+                       "group_size": G, "capacity_per_gpu": table.shard_capacity(0),
+                       "parallelism": f"keyspace-shard{world}" if world > 1 else "single",
+                       "l2": "inputs (2 x 2^%d x 4 B) and table exceed the 126 MB L2; no flush" % args.n_log2},
+            "insert_gops": n * world / (ins_ms * 1e-3) / 1e9,
+            "query_gops": n * world / (qry_ms * 1e-3) / 1e9,
+            "fill_ms": t_ms - ins_ms - qry_ms,
+            "roofline": roofline, "cpu_baseline": cpu,
+            "clocks": clk.summary(), "e2e": e2e, "gpu_launches": launches,
+            "gpu_launches_per_step": launches / args.steps,
+        }
+        print(json.dumps(line), flush=True)
+        for l in sweep_lines:
+            print(json.dumps(l), flush=True)
+    table.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_sweep(args, wd, gg, torch):
+    """config 2 sweep (alpha x |g|): insert and retrieve G ops/s with sector-roofline
+    fractions; extra lines, not the headline."""
+    out = []
+    n = 1 << args.n_log2
+    keys = gg.unique_keys(n, KEY_SEED)
+    vals = gg.values(n, VAL_SEED)
+    vout = torch.empty(n, dtype=torch.int32, device="cuda")
+    fout = torch.empty(n, dtype=torch.uint8, device="cuda")
+    hbm, _ = peaks()
+    s = torch.cuda.current_stream()
+    for alpha in (0.8, 0.9, 0.95, 0.99):
+        for G in (1, 2, 4, 8, 16, 32):
+            with wd.Table(int(math.ceil(n / alpha)), 1, G) as t:
+                ti, tq = [], []
+                for it in range(4):
+                    a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+                    t.clear(s)
+                    a.record(s)
+                    t.insert(keys, vals, s)
+                    b.record(s)
+                    t.retrieve(keys, vout, fout, s)
+                    c.record(s)
+                    torch.cuda.synchronize()
+                    if it:
+                        ti.append(a.elapsed_time(b))
+                        tq.append(b.elapsed_time(c))
+                assert t.sync() == 0
+                pc = probe_cost(alpha, G)
+                ims, qms = sum(ti) / len(ti), sum(tq) / len(tq)
+                out.append({"sweep": "config2", "alpha": alpha, "G": G,
+                            "insert_gops": n / ims / 1e6, "query_gops": n / qms / 1e6,
+                            "insert_frac": n * (40 + 32 * pc["ins_sectors"]) / (ims * 1e-3) / 1e9 / hbm,
+                            "query_frac": n * (9 + 32 * pc["hit_sectors"]) / (qms * 1e-3) / 1e9 / hbm})
+    return out
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,158 @@
+/* =====================================================================================
+ * warpdrive.h — C-ABI of the B200-native WarpDrive hot path (libwarpdrive.so).
+ *
+ * Bulk insert / retrieve of 32-bit keys and 32-bit values in an open-addressing GPU hash
+ * table with subwarp window probing (D. Jünger, C. Hundt, B. Schmidt, "WarpDrive:
+ * Massively Parallel Hashing on Multi-GPU Nodes", IPDPS 2018; P:N = line N of PAPER.md).
+ *
+ *   problem statement ...... exact map f: K -> V, k -> v
+ *   data layout ............ 4-byte key + 4-byte value packed in one 64-bit slot
+ *   load factor ............ alpha = n / c, fixed capacity
+ *   probing ................ Fig. 3 INSERT with a coalesced group of |g| lanes
+ *   duplicates ............. an existing key's value is updated
+ *   multi-GPU .............. multisplit -> transposition -> insert / query
+ *   out-of-core ............ host batches overlapped with the device cascade   (Fig. 5)
+ *
+ * No C++ or torch type crosses this boundary: plain pointers (host or device), sizes and
+ * cudaStream_t.  Everything behind wd_table_t is owned by the library.
+ *
+ * Conventions (apply to every call unless stated otherwise)
+ * ---------------------------------------------------------
+ * Errors   Argument/allocation errors are returned synchronously.  Device-side conditions
+ *          (WD_ERR_TABLE_FULL, WD_ERR_RESERVED_KEY, WD_ERR_EXCHANGE) are STICKY: they are
+ *          reported by the next call, by wd_sync() or wd_size(), and cleared by wd_clear().
+ *          wd_last_error_message() returns a thread-local human-readable description.
+ * Async    Calls enqueue work ordered after `stream` and return; `stream` is made to wait
+ *          for the call's completion, so completion is observed through `stream`.  Buffers
+ *          passed in must stay valid and unmodified until `stream` passes the call.
+ *          stream may be 0 (legacy default stream) or any stream of the table's device.
+ * Pointers Host pointers (pinned or pageable) are accepted by every mode and are streamed
+ *          in batches; pageable memory is staged through internal pinned buffers.
+ *          Device pointers must be on the table's device (single / rank / loopback modes).
+ * Threads  A handle is not thread-safe: one host thread uses it at a time.
+ * ===================================================================================== */
+#ifndef WARPDRIVE_H
+#define WARPDRIVE_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* wd_stream_t;   /* == cudaStream_t, without including CUDA */
+typedef struct wd_table wd_table_t;        /* opaque */
+
+typedef enum {
+    WD_OK = 0,
+    WD_ERR_INVALID_ARG = 1,
+    WD_ERR_OUT_OF_MEMORY = 2,
+    WD_ERR_CUDA = 3,
+    WD_ERR_NCCL = 4,
+    WD_ERR_TABLE_FULL = 5,     /* >=1 insert exhausted p_max regions (Fig. 3 Line 26);
+                                  that pair was dropped */
+    WD_ERR_RESERVED_KEY = 6,   /* >=1 input key == WD_EMPTY_KEY; those pairs were skipped
+                                  (inserts) or reported not-found (queries) */
+    WD_ERR_EXCHANGE = 7,       /* multi-GPU exchange: receive-region overflow or a peer
+                                  signal timed out */
+    WD_ERR_UNSUPPORTED = 8
+} wd_status_t;
+
+/* "empty placeholder".  Reading C8: all-ones key; never stored. */
+#define WD_EMPTY_KEY 0xFFFFFFFFu
+/* value written to vals_out[i] when found_out[i] == 0 (found_out is authoritative:
+ * stored values may legitimately equal 0xFFFFFFFF, "arbitrary 4-byte values"). */
+#define WD_NOT_FOUND 0xFFFFFFFFu
+
+/* ------------------------------------------------------------------ creation ------- */
+
+/* Single process.  n_gpus == 1: one table on the current CUDA device.
+ * n_gpus > 1: one shard per device 0..n_gpus-1, keys owned by shard p(k),
+ * peer access over NVLink; host input is split into n_gpus contiguous chunks.
+ * capacity: total slots c (alpha = n / c).  Each shard gets ceil(c / m) slots,
+ * rounded up to a multiple of 4 and to at least 32 (the 32-slot region, Fig. 3 Line 6).
+ * group_size: |g| in {1,2,4,8,16,32}.  Returns NULL on error (see wd_last_error). */
+wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size);
+
+/* Test backend: m virtual shards on the CURRENT device, running the full multi-GPU
+ * cascade (multisplit -> transposition -> insert/query -> reverse) with peer pointers
+ * that happen to be local.  Semantics identical to wd_create(capacity, m, g). */
+wd_table_t* wd_create_loopback(uint64_t capacity, int n_shards, int group_size);
+
+/* One process per GPU (torchrun).  Rank 0 calls wd_get_unique_id and the 128 bytes are
+ * broadcast by the caller (torch.distributed); every rank then calls wd_create_rank on
+ * its current device.  Collective: all ranks must call every wd_insert / wd_retrieve /
+ * wd_clear / wd_size / wd_destroy in the same order (each with its own local n >= 0). */
+wd_status_t wd_get_unique_id(uint8_t unique_id[128]);
+wd_table_t* wd_create_rank(uint64_t capacity, int rank, int world, const uint8_t unique_id[128],
+                           int group_size);
+
+/* NULL-safe.  Synchronizes, then frees table, buffers, peer mappings and communicators. */
+void wd_destroy(wd_table_t* t);
+
+/* ------------------------------------------------------------------ the hot path --- */
+
+/* a1: re-fill every slot with EMPTY and zero the counters (a fresh table). */
+wd_status_t wd_clear(wd_table_t* t, wd_stream_t stream);
+
+/* a2+a3 (and a6-a9 when m > 1, a11 for host pointers): bulk upsert of n pairs
+ * keys[i] -> vals[i] (SoA uint32 arrays).  Duplicate keys: the stored value is one of
+ * the values inserted for that key; across stream-ordered calls the later call
+ * wins.  Reserved key WD_EMPTY_KEY: skipped, sticky WD_ERR_RESERVED_KEY. */
+wd_status_t wd_insert(wd_table_t* t, const uint32_t* keys, const uint32_t* vals, uint64_t n,
+                      wd_stream_t stream);
+
+/* a4 (and a6-a10 when m > 1, a11 for host pointers): for each i, found_out[i] = 1 and
+ * vals_out[i] = the stored value if keys[i] is present, else found_out[i] = 0 and
+ * vals_out[i] = WD_NOT_FOUND.  Results in input order.  vals_out may be NULL (presence
+ * only); found_out may be NULL. */
+wd_status_t wd_retrieve(wd_table_t* t, const uint32_t* keys, uint32_t* vals_out,
+                        uint8_t* found_out, uint64_t n, wd_stream_t stream);
+
+/* a5: number of distinct keys stored (summed over shards and ranks).  Synchronizes.
+ * UINT64_MAX on error. */
+uint64_t wd_size(wd_table_t* t);
+
+/* physical slots summed over all shards (load = wd_size / wd_capacity). */
+uint64_t wd_capacity(wd_table_t* t);
+
+/* Wait for all enqueued work; returns (and keeps) sticky device-side errors. */
+wd_status_t wd_sync(wd_table_t* t);
+
+/* ------------------------------------------------------------------ options -------- */
+typedef enum {
+    WD_OPT_GROUP_SIZE = 0,   /* |g|; the probe sequence does not depend on it */
+    WD_OPT_P_MAX = 1,        /* outer probing bound p_max (Fig. 3 Line 4), default 1024 (C4) */
+    WD_OPT_BATCH = 2,        /* items per shard per pipeline batch (2^24) */
+    WD_OPT_SERIAL = 3,       /* 1: one probing group, one key at a time (deterministic
+                                layout, test hook for the Fig. 3 replay) */
+    WD_OPT_KEYS_IN_FLIGHT = 4, /* 0 = default; else keys per group in flight (4 or 8) */
+    WD_OPT_PART_SEED = 5,    /* seed of the partition function p(k) (C15) */
+    WD_OPT_PART_MODE = 6,    /* 0: p(k) = fmix32(k+seed)*m >> 32; 1: k mod m (Fig. 4) */
+    WD_OPT_N_SHARDS = 100,   /* read-only: m */
+    WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
+    WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */
+    WD_OPT_LAUNCHES = 103    /* read-only: kernels launched by the library so far */
+} wd_option_t;
+
+wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t value);
+int64_t     wd_get_option(wd_table_t* t, wd_option_t opt);   /* INT64_MIN on error */
+
+/* ------------------------------------------------------------------ diagnostics ---- */
+wd_status_t wd_last_error(void);
+const char* wd_error_string(wd_status_t s);
+const char* wd_last_error_message(void);
+
+/* slots of local shard `shard` (0-based among this process's shards) */
+uint64_t    wd_shard_capacity(wd_table_t* t, int shard);
+/* copy the raw 64-bit slots of a local shard to host memory (debug / layout tests);
+ * word = key | (uint64_t)value << 32, empty = all ones.  Synchronizes. */
+wd_status_t wd_dump(wd_table_t* t, int shard, uint64_t* host_out);
+/* per-shard device counters: [0] new keys, [1] failed inserts, [2] reserved keys,
+ * [3] exchange errors.  Synchronizes. */
+wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[4]);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* WARPDRIVE_H */

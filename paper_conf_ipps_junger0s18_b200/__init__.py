@@ -1,0 +1,233 @@
+"""paper_conf_ipps_junger0s18_b200 — B200-native WarpDrive hot path (Python binding).
+
+A thin ctypes binding over libwarpdrive.so (C-ABI in include/warpdrive.h): argument
+marshalling only.  Every step of the hot path runs in the library's sm_100a kernels;
+there is NO CPU fallback — importing this package without the built library raises.
+
+    import paper_conf_ipps_junger0s18_b200 as wd
+    t = wd.Table(capacity=int(n / 0.95), group_size=4)
+    t.insert(keys, vals)                   # torch tensors (cuda or pinned cpu) or numpy
+    vals_out, found = t.retrieve(queries)
+
+The module-level functions carry the C names (wd_create, wd_insert, ...) and take raw
+integers (pointers, stream handles); `Table` adds tensor/array marshalling.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libwarpdrive.so")
+
+WD_OK, WD_ERR_INVALID_ARG, WD_ERR_OUT_OF_MEMORY, WD_ERR_CUDA, WD_ERR_NCCL = 0, 1, 2, 3, 4
+WD_ERR_TABLE_FULL, WD_ERR_RESERVED_KEY, WD_ERR_EXCHANGE, WD_ERR_UNSUPPORTED = 5, 6, 7, 8
+WD_EMPTY_KEY = 0xFFFFFFFF
+WD_NOT_FOUND = 0xFFFFFFFF
+
+WD_OPT_GROUP_SIZE, WD_OPT_P_MAX, WD_OPT_BATCH, WD_OPT_SERIAL = 0, 1, 2, 3
+WD_OPT_KEYS_IN_FLIGHT, WD_OPT_PART_SEED, WD_OPT_PART_MODE = 4, 5, 6
+WD_OPT_N_SHARDS, WD_OPT_RANK, WD_OPT_LOCAL_SHARDS, WD_OPT_LAUNCHES = 100, 101, 102, 103
+
+EXPORTS = ["wd_create", "wd_create_loopback", "wd_get_unique_id", "wd_create_rank",
+           "wd_destroy", "wd_clear", "wd_insert", "wd_retrieve", "wd_size", "wd_capacity",
+           "wd_sync", "wd_set_option", "wd_get_option", "wd_last_error", "wd_error_string",
+           "wd_last_error_message", "wd_shard_capacity", "wd_dump", "wd_counters"]
+
+
+class WarpDriveError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{_name(status)}: {msg}")
+        self.status = status
+
+
+def _name(s):
+    try:
+        return _lib.wd_error_string(s).decode()
+    except Exception:  # pragma: no cover
+        return str(s)
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run `python __graft_entry__.py build` "
+                          "(or paper_conf_ipps_junger0s18_b200/build.py); there is no fallback")
+    L = C.CDLL(LIB_PATH)
+    u64, i32, p, i64 = C.c_uint64, C.c_int, C.c_void_p, C.c_int64
+    sig = {
+        "wd_create": ([u64, i32, i32], p),
+        "wd_create_loopback": ([u64, i32, i32], p),
+        "wd_get_unique_id": ([p], i32),
+        "wd_create_rank": ([u64, i32, i32, p, i32], p),
+        "wd_destroy": ([p], None),
+        "wd_clear": ([p, p], i32),
+        "wd_insert": ([p, p, p, u64, p], i32),
+        "wd_retrieve": ([p, p, p, p, u64, p], i32),
+        "wd_size": ([p], u64),
+        "wd_capacity": ([p], u64),
+        "wd_sync": ([p], i32),
+        "wd_set_option": ([p, i32, i64], i32),
+        "wd_get_option": ([p, i32], i64),
+        "wd_last_error": ([], i32),
+        "wd_error_string": ([i32], C.c_char_p),
+        "wd_last_error_message": ([], C.c_char_p),
+        "wd_shard_capacity": ([p, i32], u64),
+        "wd_dump": ([p, i32, p], i32),
+        "wd_counters": ([p, i32, p], i32),
+    }
+    for name, (args, res) in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = res
+    return L
+
+
+_lib = _load()
+
+# C-named thin wrappers (raw ints: pointers and cudaStream_t handles)
+for _n in EXPORTS:
+    globals()[_n] = getattr(_lib, _n)
+
+
+def _check(status: int):
+    if status != WD_OK:
+        raise WarpDriveError(status, _lib.wd_last_error_message().decode())
+
+
+def _addr(x):
+    """(pointer, nelem, is_cuda) of a torch tensor / numpy array / None."""
+    if x is None:
+        return None, 0, False
+    if isinstance(x, np.ndarray):
+        assert x.flags.c_contiguous
+        return x.ctypes.data, x.size, False
+    import torch
+    if isinstance(x, torch.Tensor):
+        assert x.is_contiguous()
+        return x.data_ptr(), x.numel(), x.is_cuda
+    raise TypeError(f"unsupported buffer type {type(x)}")
+
+
+def _stream(stream, dev_hint=None):
+    if stream is None:
+        import torch
+        if not torch.cuda.is_available():
+            return 0
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+class Table:
+    """One WarpDrive hash table (single GPU, loopback shards, single-process multi-GPU or
+    one shard per rank).  All methods are asynchronous on `stream` except size/sync/dump."""
+
+    def __init__(self, capacity: int, n_gpus: int = 1, group_size: int = 4, *,
+                 loopback_shards: int | None = None, rank: int | None = None,
+                 world: int | None = None, unique_id: bytes | None = None):
+        if loopback_shards is not None:
+            h = _lib.wd_create_loopback(int(capacity), int(loopback_shards), int(group_size))
+        elif rank is not None:
+            assert world is not None and unique_id is not None and len(unique_id) == 128
+            buf = (C.c_uint8 * 128).from_buffer_copy(unique_id)
+            h = _lib.wd_create_rank(int(capacity), int(rank), int(world), C.addressof(buf),
+                                    int(group_size))
+        else:
+            h = _lib.wd_create(int(capacity), int(n_gpus), int(group_size))
+        if not h:
+            raise WarpDriveError(_lib.wd_last_error(), _lib.wd_last_error_message().decode())
+        self._h = h
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = (C.c_uint8 * 128)()
+        _check(_lib.wd_get_unique_id(C.addressof(buf)))
+        return bytes(buf)
+
+    # -- lifetime
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.wd_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        self.close()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    @property
+    def handle(self):
+        return self._h
+
+    # -- hot path
+    def clear(self, stream=None):
+        _check(_lib.wd_clear(self._h, _stream(stream)))
+
+    def insert(self, keys, vals, stream=None):
+        kp, n, kc = _addr(keys)
+        vp, nv, vc = _addr(vals)
+        if n != nv:
+            raise ValueError("keys and vals differ in length")
+        _check(_lib.wd_insert(self._h, kp, vp, n, _stream(stream)))
+
+    def retrieve(self, keys, vals_out=None, found_out=None, stream=None):
+        kp, n, kc = _addr(keys)
+        if vals_out is None and found_out is None:
+            import torch
+            dev = keys.device if isinstance(keys, torch.Tensor) else None
+            if dev is not None:
+                pin = dev.type == "cpu" and keys.is_pinned()
+                vals_out = torch.empty(n, dtype=torch.int32, device=dev, pin_memory=pin)
+                found_out = torch.empty(n, dtype=torch.uint8, device=dev, pin_memory=pin)
+            else:
+                vals_out = np.empty(n, np.uint32)
+                found_out = np.empty(n, np.uint8)
+        vp, _, _ = _addr(vals_out)
+        fp, _, _ = _addr(found_out)
+        _check(_lib.wd_retrieve(self._h, kp, vp, fp, n, _stream(stream)))
+        return vals_out, found_out
+
+    # -- queries of state
+    def size(self) -> int:
+        s = _lib.wd_size(self._h)
+        if s == 2**64 - 1:
+            _check(_lib.wd_last_error() or WD_ERR_CUDA)
+        return int(s)
+
+    def capacity(self) -> int:
+        return int(_lib.wd_capacity(self._h))
+
+    def sync(self) -> int:
+        """Wait; returns the sticky device-side status (0 = WD_OK) without raising."""
+        return int(_lib.wd_sync(self._h))
+
+    def set_option(self, opt: int, value: int):
+        _check(_lib.wd_set_option(self._h, int(opt), int(value)))
+
+    def get_option(self, opt: int) -> int:
+        return int(_lib.wd_get_option(self._h, int(opt)))
+
+    def shard_capacity(self, shard: int = 0) -> int:
+        return int(_lib.wd_shard_capacity(self._h, shard))
+
+    def dump(self, shard: int = 0) -> np.ndarray:
+        out = np.empty(self.shard_capacity(shard), np.uint64)
+        _check(_lib.wd_dump(self._h, shard, out.ctypes.data))
+        return out
+
+    def counters(self, shard: int = 0) -> dict:
+        out = np.zeros(4, np.uint64)
+        _check(_lib.wd_counters(self._h, shard, out.ctypes.data))
+        return {"new": int(out[0]), "failed": int(out[1]), "reserved": int(out[2]),
+                "exchange_errors": int(out[3])}
+
+    @property
+    def launches(self) -> int:
+        return self.get_option(WD_OPT_LAUNCHES)

@@ -1,0 +1,1119 @@
+// =====================================================================================
+// warpdrive.cu — host side of libwarpdrive.so: the C-ABI of include/warpdrive.h.
+//
+//   wd_table ........ m shards ("GPU i exclusively holds keys where p(k) = i"),
+//                     of which this process owns 1 (single / rank mode) or all
+//                     (loopback: m virtual shards on one device; multi: one per device).
+//   single path ..... device input: one probe kernel on the caller's stream.
+//                     host input: out-of-core pipeline H2D(b+1) || probe(b) || D2H(b-1)
+//                     on three streams with double-buffered staging (Fig. 5).
+//   cascade (m > 1) . per batch: multisplit fused with the push into the owners'
+//                     receive regions -> publish T row + ready flags -> owner waits for its
+//                     T column -> local insert / query -> done flags -> (query) origin
+//                     pulls results back and unpermutes -> consumed flags.  All signalling
+//                     is device-side (no host synchronisation per batch); receive and
+//                     result regions are double-buffered by epoch parity.
+// =====================================================================================
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <unordered_map>
+#include <vector>
+
+#include "../../include/warpdrive.h"
+#include "wd_device.cuh"
+
+namespace {
+
+thread_local wd_status_t g_last = WD_OK;
+thread_local char g_msg[1024] = "";
+
+wd_status_t fail(wd_status_t s, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_msg, sizeof g_msg, fmt, ap);
+  va_end(ap);
+  g_last = s;
+  return s;
+}
+
+#define CK(x)                                                                            \
+  do {                                                                                   \
+    cudaError_t e_ = (x);                                                                \
+    if (e_ != cudaSuccess)                                                               \
+      return fail(e_ == cudaErrorMemoryAllocation ? WD_ERR_OUT_OF_MEMORY : WD_ERR_CUDA,  \
+                  "%s: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, __LINE__);     \
+  } while (0)
+#define NK(x)                                                                            \
+  do {                                                                                   \
+    ncclResult_t r_ = (x);                                                               \
+    if (r_ != ncclSuccess)                                                               \
+      return fail(WD_ERR_NCCL, "%s: %s (%s:%d)", #x, ncclGetErrorString(r_), __FILE__,   \
+                  __LINE__);                                                             \
+  } while (0)
+#define TRY(x)                          \
+  do {                                  \
+    wd_status_t s_ = (x);               \
+    if (s_ != WD_OK) return s_;         \
+  } while (0)
+
+enum Mode { MODE_SINGLE = 0, MODE_LOOPBACK = 1, MODE_MULTI = 2, MODE_RANK = 3 };
+enum Flag { FLAG_READY = 0, FLAG_DONE = 1, FLAG_RESC = 2, FLAG_N = 3 };
+enum PtrKind { PK_DEVICE = 0, PK_PINNED = 1, PK_PAGEABLE = 2 };
+
+constexpr unsigned long long kWaitTimeoutNs = 30ull * 1000 * 1000 * 1000;  // 30 s
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int d) {
+    cudaGetDevice(&prev);
+    if (prev != d) cudaSetDevice(d);
+  }
+  ~DeviceGuard() {
+    int cur;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+// pointers into one shard's exchange arena, valid in this process (own or peer-mapped)
+struct PeerView {
+  unsigned long long* recv[2] = {nullptr, nullptr};        // [m][B] items written by senders
+  unsigned long long* res[2] = {nullptr, nullptr};         // [m][B] packed query results
+  unsigned long long* recv_count[2] = {nullptr, nullptr};  // [m] column of T
+  unsigned long long* flags = nullptr;                     // [FLAG_N][m]
+};
+
+struct Shard {
+  int id = 0;        // global shard index (= owner id of p(k))
+  int device = 0;
+  uint64_t cap = 0, nb = 0;
+  unsigned long long* slots = nullptr;
+  unsigned long long* counters = nullptr;
+  cudaStream_t s_main = nullptr, s_h2d = nullptr, s_d2h = nullptr;
+  bool own_main = true;
+  // exchange arena (one allocation: IPC-exportable)
+  void* arena = nullptr;
+  size_t arena_bytes = 0;
+  PeerView self;
+  unsigned long long* cursor[2] = {nullptr, nullptr};  // [m] local send counters
+  uint32_t* pos[2] = {nullptr, nullptr};               // [B] query positions
+  // staging for host input / output
+  uint64_t st_batch = 0;
+  uint32_t *st_keys[2] = {}, *st_vals[2] = {}, *st_vout[2] = {};
+  uint8_t* st_fout[2] = {};
+  uint64_t pin_batch = 0;
+  uint32_t *pin_keys[2] = {}, *pin_vals[2] = {}, *pin_vout[2] = {};
+  uint8_t* pin_fout[2] = {};
+  cudaEvent_t ev_h2d[2] = {}, ev_free[2] = {}, ev_kdone[2] = {}, ev_d2h[2] = {};
+  cudaEvent_t ev_join_main = nullptr, ev_join_h2d = nullptr, ev_join_d2h = nullptr;
+  bool h2d_pending[2] = {false, false}, d2h_pending[2] = {false, false};
+};
+
+}  // namespace
+
+struct wd_table {
+  int mode = MODE_SINGLE;
+  int m = 1;          // number of shards (= GPUs, or virtual shards in loopback)
+  int rank = 0;       // rank mode: this process's shard id
+  int G = 4;
+  int pmax = 1024;
+  int kif = 0;        // keys in flight per group (0 = default)
+  uint64_t batch = 1ull << 24;
+  int serial = 0;
+  uint32_t pseed = 0x9E3779B9u;
+  int pmode = 0;
+  unsigned long long epoch = 0;
+  unsigned long long res_used[2] = {0, 0};  // last (query) epoch that filled result slot i
+  uint64_t launches = 0;
+  uint64_t xbatch = 0;  // batch size the exchange arenas were built for
+  int sm_count = 148;
+  std::vector<Shard> local;
+  std::vector<PeerView> peers;  // size m
+  std::vector<void*> opened;    // IPC-mapped peer arenas (rank mode)
+  ncclComm_t comm = nullptr;
+  unsigned long long* d_scratch = nullptr;  // rank mode: allreduce scratch
+  cudaStream_t loop_stream = nullptr;       // loopback: one stream for all shards
+};
+
+namespace {
+
+// ------------------------------------------------------------------ helpers
+uint64_t round_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+PtrKind classify(const void* p, int* dev) {
+  if (!p) return PK_DEVICE;
+  cudaPointerAttributes a;
+  cudaError_t e = cudaPointerGetAttributes(&a, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return PK_PAGEABLE;
+  }
+  if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
+    if (dev) *dev = a.device;
+    return PK_DEVICE;
+  }
+  if (a.type == cudaMemoryTypeHost) return PK_PINNED;
+  return PK_PAGEABLE;
+}
+
+template <class K>
+int blocks_per_sm(K kern) {
+  static std::unordered_map<const void*, int> cache;
+  auto it = cache.find((const void*)kern);
+  if (it != cache.end()) return it->second;
+  int nb = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, wd::kBlock, 0) != cudaSuccess) {
+    cudaGetLastError();
+    nb = 1;
+  }
+  nb = std::max(nb, 1);
+  cache[(const void*)kern] = nb;
+  return nb;
+}
+
+// ------------------------------------------------------------------ probe dispatch
+template <int G, int K, bool INSERT, class In, class Out>
+wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
+                           cudaStream_t st) {
+  auto kern = wd::probe_kernel<G, K, INSERT, In, Out>;
+  const wd::TableView tv{s.slots, s.nb, static_cast<uint32_t>(t->pmax)};
+  int grid = 1, block = 32;
+  if (!t->serial) {
+    block = wd::kBlock;
+    const uint64_t keys_per_block = uint64_t(wd::kBlock / 32) * K * (32 / G);
+    const uint64_t need = std::max<uint64_t>(1, (n_hint + keys_per_block - 1) / keys_per_block);
+    grid = static_cast<int>(std::min<uint64_t>(need, uint64_t(t->sm_count) * blocks_per_sm(kern)));
+  }
+  kern<<<grid, block, 0, st>>>(tv, in, out, s.counters, t->serial);
+  CK(cudaGetLastError());
+  t->launches++;
+  return WD_OK;
+}
+
+template <int G, bool INSERT, class In, class Out>
+wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
+                           cudaStream_t st) {
+  int k = t->kif;
+  if (k == 0) k = (G <= 2) ? 4 : 8;
+  if (k == 4) return launch_probe_k<G, 4, INSERT>(t, s, in, out, n_hint, st);
+  return launch_probe_k<G, 8, INSERT>(t, s, in, out, n_hint, st);
+}
+
+template <bool INSERT, class In, class Out>
+wd_status_t launch_probe(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
+                         cudaStream_t st) {
+  switch (t->G) {
+    case 1: return launch_probe_g<1, INSERT>(t, s, in, out, n_hint, st);
+    case 2: return launch_probe_g<2, INSERT>(t, s, in, out, n_hint, st);
+    case 4: return launch_probe_g<4, INSERT>(t, s, in, out, n_hint, st);
+    case 8: return launch_probe_g<8, INSERT>(t, s, in, out, n_hint, st);
+    case 16: return launch_probe_g<16, INSERT>(t, s, in, out, n_hint, st);
+    case 32: return launch_probe_g<32, INSERT>(t, s, in, out, n_hint, st);
+  }
+  return fail(WD_ERR_INVALID_ARG, "group size %d not in {1,2,4,8,16,32}", t->G);
+}
+
+// ------------------------------------------------------------------ shard lifetime
+wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
+                       cudaStream_t shared_main) {
+  DeviceGuard g(device);
+  s.id = id;
+  s.device = device;
+  s.cap = cap;
+  s.nb = (cap - 32) / 4 + 1;
+  CK(cudaMalloc(&s.slots, cap * sizeof(unsigned long long)));
+  CK(cudaMalloc(&s.counters, wd::CNT_N * sizeof(unsigned long long)));
+  if (shared_main) {
+    s.s_main = shared_main;
+    s.own_main = false;
+  } else {
+    CK(cudaStreamCreateWithFlags(&s.s_main, cudaStreamNonBlocking));
+  }
+  CK(cudaStreamCreateWithFlags(&s.s_h2d, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&s.s_d2h, cudaStreamNonBlocking));
+  for (int i = 0; i < 2; ++i) {
+    CK(cudaEventCreateWithFlags(&s.ev_h2d[i], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&s.ev_free[i], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&s.ev_kdone[i], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&s.ev_d2h[i], cudaEventDisableTiming));
+  }
+  CK(cudaEventCreateWithFlags(&s.ev_join_main, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&s.ev_join_h2d, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&s.ev_join_d2h, cudaEventDisableTiming));
+  // a1: fresh table
+  const int grid = t->sm_count * 4;
+  wd::fill_kernel<<<grid, wd::kBlock, 0, s.s_main>>>(s.slots, s.cap, s.counters, wd::CNT_N);
+  CK(cudaGetLastError());
+  t->launches++;
+  CK(cudaStreamSynchronize(s.s_main));  // device-path calls use the caller's stream
+  return WD_OK;
+}
+
+void free_exchange(Shard& s) {
+  DeviceGuard g(s.device);
+  if (s.arena) cudaFree(s.arena);
+  s.arena = nullptr;
+  s.self = PeerView{};
+  for (int i = 0; i < 2; ++i) {
+    if (s.cursor[i]) cudaFree(s.cursor[i]);
+    if (s.pos[i]) cudaFree(s.pos[i]);
+    s.cursor[i] = nullptr;
+    s.pos[i] = nullptr;
+  }
+}
+
+void free_staging(Shard& s) {
+  DeviceGuard g(s.device);
+  for (int i = 0; i < 2; ++i) {
+    if (s.st_keys[i]) cudaFree(s.st_keys[i]);
+    if (s.st_vals[i]) cudaFree(s.st_vals[i]);
+    if (s.st_vout[i]) cudaFree(s.st_vout[i]);
+    if (s.st_fout[i]) cudaFree(s.st_fout[i]);
+    if (s.pin_keys[i]) cudaFreeHost(s.pin_keys[i]);
+    if (s.pin_vals[i]) cudaFreeHost(s.pin_vals[i]);
+    if (s.pin_vout[i]) cudaFreeHost(s.pin_vout[i]);
+    if (s.pin_fout[i]) cudaFreeHost(s.pin_fout[i]);
+    s.st_keys[i] = s.st_vals[i] = s.st_vout[i] = nullptr;
+    s.st_fout[i] = nullptr;
+    s.pin_keys[i] = s.pin_vals[i] = s.pin_vout[i] = nullptr;
+    s.pin_fout[i] = nullptr;
+  }
+  s.st_batch = s.pin_batch = 0;
+}
+
+void shard_free(Shard& s) {
+  DeviceGuard g(s.device);
+  if (s.s_main) cudaStreamSynchronize(s.s_main);
+  if (s.s_h2d) cudaStreamSynchronize(s.s_h2d);
+  if (s.s_d2h) cudaStreamSynchronize(s.s_d2h);
+  free_exchange(s);
+  free_staging(s);
+  if (s.slots) cudaFree(s.slots);
+  if (s.counters) cudaFree(s.counters);
+  for (int i = 0; i < 2; ++i) {
+    if (s.ev_h2d[i]) cudaEventDestroy(s.ev_h2d[i]);
+    if (s.ev_free[i]) cudaEventDestroy(s.ev_free[i]);
+    if (s.ev_kdone[i]) cudaEventDestroy(s.ev_kdone[i]);
+    if (s.ev_d2h[i]) cudaEventDestroy(s.ev_d2h[i]);
+  }
+  if (s.ev_join_main) cudaEventDestroy(s.ev_join_main);
+  if (s.ev_join_h2d) cudaEventDestroy(s.ev_join_h2d);
+  if (s.ev_join_d2h) cudaEventDestroy(s.ev_join_d2h);
+  if (s.own_main && s.s_main) cudaStreamDestroy(s.s_main);
+  if (s.s_h2d) cudaStreamDestroy(s.s_h2d);
+  if (s.s_d2h) cudaStreamDestroy(s.s_d2h);
+  s = Shard{};
+}
+
+wd_status_t ensure_staging(Shard& s, uint64_t B, bool pageable) {
+  DeviceGuard g(s.device);
+  if (s.st_batch < B) {
+    for (int i = 0; i < 2; ++i) {
+      if (s.st_keys[i]) cudaFree(s.st_keys[i]);
+      if (s.st_vals[i]) cudaFree(s.st_vals[i]);
+      if (s.st_vout[i]) cudaFree(s.st_vout[i]);
+      if (s.st_fout[i]) cudaFree(s.st_fout[i]);
+      CK(cudaMalloc(&s.st_keys[i], B * 4));
+      CK(cudaMalloc(&s.st_vals[i], B * 4));
+      CK(cudaMalloc(&s.st_vout[i], B * 4));
+      CK(cudaMalloc(&s.st_fout[i], B));
+    }
+    s.st_batch = B;
+  }
+  if (pageable && s.pin_batch < B) {
+    for (int i = 0; i < 2; ++i) {
+      if (s.pin_keys[i]) cudaFreeHost(s.pin_keys[i]);
+      if (s.pin_vals[i]) cudaFreeHost(s.pin_vals[i]);
+      if (s.pin_vout[i]) cudaFreeHost(s.pin_vout[i]);
+      if (s.pin_fout[i]) cudaFreeHost(s.pin_fout[i]);
+      CK(cudaMallocHost(&s.pin_keys[i], B * 4));
+      CK(cudaMallocHost(&s.pin_vals[i], B * 4));
+      CK(cudaMallocHost(&s.pin_vout[i], B * 4));
+      CK(cudaMallocHost(&s.pin_fout[i], B));
+    }
+    s.pin_batch = B;
+  }
+  return WD_OK;
+}
+
+// arena layout: recv[2] | res[2] | recv_count[2] | flags
+PeerView arena_view(void* base, int m, uint64_t B) {
+  PeerView v;
+  char* p = static_cast<char*>(base);
+  const size_t region = size_t(m) * B * 8;
+  for (int i = 0; i < 2; ++i) v.recv[i] = reinterpret_cast<unsigned long long*>(p + i * region);
+  p += 2 * region;
+  for (int i = 0; i < 2; ++i) v.res[i] = reinterpret_cast<unsigned long long*>(p + i * region);
+  p += 2 * region;
+  for (int i = 0; i < 2; ++i) v.recv_count[i] = reinterpret_cast<unsigned long long*>(p + i * m * 8);
+  p += 2 * m * 8;
+  v.flags = reinterpret_cast<unsigned long long*>(p);
+  return v;
+}
+size_t arena_size(int m, uint64_t B) {
+  return 4 * size_t(m) * B * 8 + 2 * size_t(m) * 8 + size_t(FLAG_N) * m * 8 + 256;
+}
+
+wd_status_t exchange_init_shard(wd_table* t, Shard& s, uint64_t B) {
+  DeviceGuard g(s.device);
+  s.arena_bytes = arena_size(t->m, B);
+  CK(cudaMalloc(&s.arena, s.arena_bytes));
+  s.self = arena_view(s.arena, t->m, B);
+  // counts and flags start at 0: epochs are >= 1
+  CK(cudaMemsetAsync(s.self.recv_count[0], 0, 2 * t->m * 8 + FLAG_N * t->m * 8, s.s_main));
+  for (int i = 0; i < 2; ++i) {
+    CK(cudaMalloc(&s.cursor[i], t->m * 8));
+    CK(cudaMemsetAsync(s.cursor[i], 0, t->m * 8, s.s_main));
+    CK(cudaMalloc(&s.pos[i], B * 4));
+  }
+  CK(cudaStreamSynchronize(s.s_main));
+  return WD_OK;
+}
+
+wd_status_t rank_allgather_views(wd_table* t, uint64_t B);
+
+// (re)build the exchange arenas for batch size B (collective in rank mode)
+wd_status_t ensure_exchange(wd_table* t) {
+  if (t->m == 1) return WD_OK;
+  if (t->xbatch == t->batch) return WD_OK;
+  const uint64_t B = t->batch;
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    CK(cudaStreamSynchronize(s.s_main));
+  }
+  for (void* p : t->opened) cudaIpcCloseMemHandle(p);
+  t->opened.clear();
+  for (auto& s : t->local) free_exchange(s);
+  for (auto& s : t->local) TRY(exchange_init_shard(t, s, B));
+  t->peers.assign(t->m, PeerView{});
+  if (t->mode == MODE_RANK) {
+    TRY(rank_allgather_views(t, B));
+  } else {
+    for (auto& s : t->local) t->peers[s.id] = s.self;
+  }
+  t->xbatch = B;
+  t->epoch = 0;  // fresh flags
+  t->res_used[0] = t->res_used[1] = 0;
+  return WD_OK;
+}
+
+wd_status_t rank_allgather_views(wd_table* t, uint64_t B) {
+  Shard& s = t->local[0];
+  DeviceGuard g(s.device);
+  cudaIpcMemHandle_t h;
+  CK(cudaIpcGetMemHandle(&h, s.arena));
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "ipc handle size");
+  char* d_buf = nullptr;
+  CK(cudaMalloc(&d_buf, size_t(64) * t->m));
+  CK(cudaMemcpy(d_buf + 64 * t->rank, &h, 64, cudaMemcpyHostToDevice));
+  NK(ncclAllGather(d_buf + 64 * t->rank, d_buf, 64, ncclChar, t->comm, s.s_main));
+  std::vector<cudaIpcMemHandle_t> all(t->m);
+  CK(cudaMemcpyAsync(all.data(), d_buf, size_t(64) * t->m, cudaMemcpyDeviceToHost, s.s_main));
+  CK(cudaStreamSynchronize(s.s_main));
+  cudaFree(d_buf);
+  for (int d = 0; d < t->m; ++d) {
+    if (d == t->rank) {
+      t->peers[d] = s.self;
+      continue;
+    }
+    void* base = nullptr;
+    CK(cudaIpcOpenMemHandle(&base, all[d], cudaIpcMemLazyEnablePeerAccess));
+    t->opened.push_back(base);
+    t->peers[d] = arena_view(base, t->m, B);
+  }
+  // everyone mapped everyone before first use
+  NK(ncclAllReduce(t->d_scratch, t->d_scratch, 1, ncclUint64, ncclSum, t->comm, s.s_main));
+  CK(cudaStreamSynchronize(s.s_main));
+  return WD_OK;
+}
+
+// ------------------------------------------------------------------ join helpers
+// make the shard's internal streams wait for `stream`
+wd_status_t fork_from(wd_table* t, cudaStream_t stream, cudaEvent_t* ev_tmp) {
+  CK(cudaEventCreateWithFlags(ev_tmp, cudaEventDisableTiming));
+  CK(cudaEventRecord(*ev_tmp, stream));
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    CK(cudaStreamWaitEvent(s.s_main, *ev_tmp, 0));
+    CK(cudaStreamWaitEvent(s.s_h2d, *ev_tmp, 0));
+    CK(cudaStreamWaitEvent(s.s_d2h, *ev_tmp, 0));
+  }
+  return WD_OK;
+}
+// make `stream` wait for all internal streams
+wd_status_t join_into(wd_table* t, cudaStream_t stream, cudaEvent_t ev_tmp) {
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    CK(cudaEventRecord(s.ev_join_main, s.s_main));
+    CK(cudaEventRecord(s.ev_join_h2d, s.s_h2d));
+    CK(cudaEventRecord(s.ev_join_d2h, s.s_d2h));
+    CK(cudaStreamWaitEvent(stream, s.ev_join_main, 0));
+    CK(cudaStreamWaitEvent(stream, s.ev_join_h2d, 0));
+    CK(cudaStreamWaitEvent(stream, s.ev_join_d2h, 0));
+  }
+  if (ev_tmp) cudaEventDestroy(ev_tmp);
+  return WD_OK;
+}
+
+// ------------------------------------------------------------------ per-shard IO chunk
+struct IO {
+  const uint32_t* keys = nullptr;
+  const uint32_t* vals = nullptr;
+  uint32_t* vout = nullptr;
+  uint8_t* fout = nullptr;
+  uint64_t n = 0;
+  PtrKind kin = PK_DEVICE, kout = PK_DEVICE;
+};
+
+// stage batch b's input of `io` into device memory; returns device pointers
+wd_status_t stage_in(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slot, bool with_vals,
+                     const uint32_t** dk, const uint32_t** dv) {
+  if (io.kin == PK_DEVICE) {
+    *dk = io.keys + off;
+    *dv = with_vals ? io.vals + off : nullptr;
+    return WD_OK;
+  }
+  DeviceGuard g(s.device);
+  if (s.h2d_pending[slot]) CK(cudaStreamWaitEvent(s.s_h2d, s.ev_free[slot], 0));
+  const uint32_t* hk = io.keys + off;
+  const uint32_t* hv = with_vals ? io.vals + off : nullptr;
+  if (io.kin == PK_PAGEABLE && cnt) {
+    // the pinned bounce buffer of this slot must not be read by an in-flight copy
+    CK(cudaEventSynchronize(s.ev_h2d[slot]));
+    memcpy(s.pin_keys[slot], hk, cnt * 4);
+    if (hv) memcpy(s.pin_vals[slot], hv, cnt * 4);
+    hk = s.pin_keys[slot];
+    hv = hv ? s.pin_vals[slot] : nullptr;
+  }
+  if (cnt) {
+    CK(cudaMemcpyAsync(s.st_keys[slot], hk, cnt * 4, cudaMemcpyHostToDevice, s.s_h2d));
+    if (hv) CK(cudaMemcpyAsync(s.st_vals[slot], hv, cnt * 4, cudaMemcpyHostToDevice, s.s_h2d));
+  }
+  CK(cudaEventRecord(s.ev_h2d[slot], s.s_h2d));
+  CK(cudaStreamWaitEvent(s.s_main, s.ev_h2d[slot], 0));
+  s.h2d_pending[slot] = true;
+  *dk = s.st_keys[slot];
+  *dv = with_vals ? s.st_vals[slot] : nullptr;
+  return WD_OK;
+}
+
+// device output pointers for batch b
+void out_ptrs(Shard& s, const IO& io, uint64_t off, int slot, uint32_t** dv, uint8_t** df) {
+  if (io.kout == PK_DEVICE) {
+    *dv = io.vout ? io.vout + off : nullptr;
+    *df = io.fout ? io.fout + off : nullptr;
+  } else {
+    *dv = io.vout ? s.st_vout[slot] : nullptr;
+    *df = io.fout ? s.st_fout[slot] : nullptr;
+  }
+}
+
+// after the kernel that consumed slot `slot` (recorded on s_main): release staging;
+// for host outputs copy results back (pageable: through the pinned bounce, synchronously)
+wd_status_t stage_out(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slot, bool query) {
+  DeviceGuard g(s.device);
+  CK(cudaEventRecord(s.ev_kdone[slot], s.s_main));
+  if (!query || io.kout == PK_DEVICE) {
+    if (io.kin != PK_DEVICE) CK(cudaEventRecord(s.ev_free[slot], s.s_main));
+    return WD_OK;
+  }
+  CK(cudaStreamWaitEvent(s.s_d2h, s.ev_kdone[slot], 0));
+  if (io.kout == PK_PINNED) {
+    if (io.vout && cnt) CK(cudaMemcpyAsync(io.vout + off, s.st_vout[slot], cnt * 4, cudaMemcpyDeviceToHost, s.s_d2h));
+    if (io.fout && cnt) CK(cudaMemcpyAsync(io.fout + off, s.st_fout[slot], cnt, cudaMemcpyDeviceToHost, s.s_d2h));
+    CK(cudaEventRecord(s.ev_free[slot], s.s_d2h));
+  } else {
+    if (io.vout && cnt) CK(cudaMemcpyAsync(s.pin_vout[slot], s.st_vout[slot], cnt * 4, cudaMemcpyDeviceToHost, s.s_d2h));
+    if (io.fout && cnt) CK(cudaMemcpyAsync(s.pin_fout[slot], s.st_fout[slot], cnt, cudaMemcpyDeviceToHost, s.s_d2h));
+    CK(cudaEventRecord(s.ev_free[slot], s.s_d2h));
+    CK(cudaEventSynchronize(s.ev_free[slot]));
+    if (io.vout) memcpy(io.vout + off, s.pin_vout[slot], cnt * 4);
+    if (io.fout) memcpy(io.fout + off, s.pin_fout[slot], cnt);
+  }
+  return WD_OK;
+}
+
+bool needs_staging(const IO& io) { return io.kin != PK_DEVICE || io.kout != PK_DEVICE; }
+
+// ------------------------------------------------------------------ single-shard path
+wd_status_t single_op(wd_table* t, bool insert, const IO& io, cudaStream_t stream) {
+  Shard& s = t->local[0];
+  DeviceGuard g(s.device);
+  if (!needs_staging(io)) {  // device-resident: one kernel on the caller's stream
+    if (io.n == 0) return WD_OK;
+    const wd::InSoA in{io.keys, io.vals, io.n};
+    if (insert) return launch_probe<true>(t, s, in, wd::OutNone{}, io.n, stream);
+    return launch_probe<false>(t, s, in, wd::OutSoA{io.vout, io.fout}, io.n, stream);
+  }
+  // out-of-core pipeline (Fig. 5): H2D(b+1) || probe(b) || D2H(b-1)
+  const uint64_t B = t->batch;
+  TRY(ensure_staging(s, B, io.kin == PK_PAGEABLE || io.kout == PK_PAGEABLE));
+  cudaEvent_t ev0;
+  TRY(fork_from(t, stream, &ev0));
+  s.h2d_pending[0] = s.h2d_pending[1] = false;
+  const uint64_t nbt = (io.n + B - 1) / B;
+  for (uint64_t b = 0; b < nbt; ++b) {
+    const int slot = int(b & 1);
+    const uint64_t off = b * B, cnt = std::min(B, io.n - off);
+    const uint32_t *dk, *dv;
+    TRY(stage_in(s, io, off, cnt, slot, insert, &dk, &dv));
+    const wd::InSoA in{dk, dv, cnt};
+    if (insert) {
+      TRY(launch_probe<true>(t, s, in, wd::OutNone{}, cnt, s.s_main));
+    } else {
+      uint32_t* ov; uint8_t* of;
+      out_ptrs(s, io, off, slot, &ov, &of);
+      TRY(launch_probe<false>(t, s, in, wd::OutSoA{ov, of}, cnt, s.s_main));
+    }
+    TRY(stage_out(s, io, off, cnt, slot, !insert));
+  }
+  return join_into(t, stream, ev0);
+}
+
+// ------------------------------------------------------------------ multi-shard cascade
+wd::FlagPtrs flag_ptrs(wd_table* t, int flag, int who) {
+  wd::FlagPtrs f{};
+  for (int d = 0; d < t->m; ++d) f.p[d] = t->peers[d].flags + flag * t->m + who;
+  return f;
+}
+
+wd_status_t launch_wait(wd_table* t, Shard& s, int flag, unsigned long long target) {
+  wd::wait_kernel<<<1, 32, 0, s.s_main>>>(s.self.flags + flag * t->m, t->m, target,
+                                          kWaitTimeoutNs, s.counters);
+  CK(cudaGetLastError());
+  t->launches++;
+  return WD_OK;
+}
+wd_status_t launch_signal(wd_table* t, Shard& s, int flag, unsigned long long epoch) {
+  wd::signal_kernel<<<1, 32, 0, s.s_main>>>(flag_ptrs(t, flag, s.id), t->m, epoch);
+  CK(cudaGetLastError());
+  t->launches++;
+  return WD_OK;
+}
+
+wd_status_t agree_batches(wd_table* t, uint64_t local_nbt, uint64_t* global_nbt) {
+  if (t->mode != MODE_RANK) {
+    *global_nbt = local_nbt;
+    return WD_OK;
+  }
+  Shard& s = t->local[0];
+  DeviceGuard g(s.device);
+  unsigned long long v = local_nbt;
+  CK(cudaMemcpyAsync(t->d_scratch, &v, 8, cudaMemcpyHostToDevice, s.s_main));
+  NK(ncclAllReduce(t->d_scratch, t->d_scratch, 1, ncclUint64, ncclMax, t->comm, s.s_main));
+  CK(cudaMemcpyAsync(&v, t->d_scratch, 8, cudaMemcpyDeviceToHost, s.s_main));
+  CK(cudaStreamSynchronize(s.s_main));
+  *global_nbt = v;
+  return WD_OK;
+}
+
+wd_status_t cascade_op(wd_table* t, bool insert, std::vector<IO>& ios, cudaStream_t stream) {
+  TRY(ensure_exchange(t));
+  const uint64_t B = t->batch;
+  const int m = t->m;
+  uint64_t local_nbt = 0;
+  for (size_t r = 0; r < t->local.size(); ++r) {
+    local_nbt = std::max(local_nbt, (ios[r].n + B - 1) / B);
+    if (needs_staging(ios[r]))
+      TRY(ensure_staging(t->local[r], B,
+                         ios[r].kin == PK_PAGEABLE || ios[r].kout == PK_PAGEABLE));
+  }
+  uint64_t nbt = 0;
+  TRY(agree_batches(t, local_nbt, &nbt));
+  if (nbt == 0) return WD_OK;
+  cudaEvent_t ev0;
+  TRY(fork_from(t, stream, &ev0));
+  for (auto& s : t->local) s.h2d_pending[0] = s.h2d_pending[1] = false;
+
+  for (uint64_t b = 0; b < nbt; ++b) {
+    const unsigned long long e = t->epoch + 1 + b;
+    const int slot = int(e & 1);
+    // ---- phase A: every local shard multisplits its batch into the owners' regions
+    for (size_t r = 0; r < t->local.size(); ++r) {
+      Shard& s = t->local[r];
+      const IO& io = ios[r];
+      DeviceGuard g(s.device);
+      const uint64_t off = std::min(io.n, b * B), cnt = std::min(B, io.n - off);
+      const uint32_t *dk = nullptr, *dv = nullptr;
+      TRY(stage_in(s, io, off, cnt, int(b & 1), insert, &dk, &dv));
+      if (e > 2) TRY(launch_wait(t, s, FLAG_DONE, e - 2));  // owners released region e-2
+      if (cnt) {
+        wd::DstPtrs dst{};
+        for (int d = 0; d < m; ++d) {
+          if (insert) dst.p[d] = t->peers[d].recv[slot] + uint64_t(s.id) * B;
+          else dst.p[d] = reinterpret_cast<uint32_t*>(t->peers[d].recv[slot]) + uint64_t(s.id) * B;
+        }
+        const uint64_t tiles = (cnt + wd::kBlock * 8 - 1) / (wd::kBlock * 8);
+        const int grid = int(std::min<uint64_t>(tiles, uint64_t(t->sm_count) * 4));
+        if (insert)
+          wd::multisplit_kernel<true><<<grid, wd::kBlock, 0, s.s_main>>>(
+              dk, dv, cnt, dst, s.cursor[slot], nullptr, m, t->pseed, t->pmode, B, s.counters);
+        else
+          wd::multisplit_kernel<false><<<grid, wd::kBlock, 0, s.s_main>>>(
+              dk, nullptr, cnt, dst, s.cursor[slot], s.pos[slot], m, t->pseed, t->pmode, B,
+              s.counters);
+        CK(cudaGetLastError());
+        t->launches++;
+      }
+      if (insert) TRY(stage_out(s, io, off, cnt, int(b & 1), false));  // input slot free
+      wd::FlagPtrs cnt_dst{};
+      for (int d = 0; d < m; ++d) cnt_dst.p[d] = t->peers[d].recv_count[slot] + s.id;
+      wd::publish_kernel<<<1, 32, 0, s.s_main>>>(s.cursor[slot], cnt_dst,
+                                                 flag_ptrs(t, FLAG_READY, s.id), m, e);
+      CK(cudaGetLastError());
+      t->launches++;
+    }
+    // ---- phase B: every local shard inserts / queries its column of T
+    for (auto& s : t->local) {
+      DeviceGuard g(s.device);
+      TRY(launch_wait(t, s, FLAG_READY, e));
+      if (insert) {
+        const wd::InSeg<true> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
+        TRY(launch_probe<true>(t, s, in, wd::OutNone{}, B, s.s_main));
+      } else {
+        // origins consumed the results of the previous query epoch that used this slot
+        if (t->res_used[slot]) TRY(launch_wait(t, s, FLAG_RESC, t->res_used[slot]));
+        const wd::InSeg<false> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
+        TRY(launch_probe<false>(t, s, in, wd::OutPacked{s.self.res[slot]}, B, s.s_main));
+      }
+      TRY(launch_signal(t, s, FLAG_DONE, e));
+    }
+    if (insert) continue;
+    t->res_used[slot] = e;
+    // ---- phase C (query): every origin pulls its results back and unpermutes
+    for (size_t r = 0; r < t->local.size(); ++r) {
+      Shard& s = t->local[r];
+      const IO& io = ios[r];
+      DeviceGuard g(s.device);
+      const uint64_t off = std::min(io.n, b * B), cnt = std::min(B, io.n - off);
+      TRY(launch_wait(t, s, FLAG_DONE, e));
+      if (cnt) {
+        wd::DstPtrs src{};
+        for (int d = 0; d < m; ++d) src.p[d] = t->peers[d].res[slot] + uint64_t(s.id) * B;
+        uint32_t* ov; uint8_t* of;
+        out_ptrs(s, io, off, int(b & 1), &ov, &of);
+        const int grid = int(std::min<uint64_t>((cnt + wd::kBlock - 1) / wd::kBlock,
+                                                uint64_t(t->sm_count) * 8));
+        wd::unpermute_kernel<<<grid, wd::kBlock, 0, s.s_main>>>(s.pos[slot], cnt, src, ov, of);
+        CK(cudaGetLastError());
+        t->launches++;
+      }
+      TRY(launch_signal(t, s, FLAG_RESC, e));
+      TRY(stage_out(s, io, off, cnt, int(b & 1), true));
+    }
+  }
+  t->epoch += nbt;
+  return join_into(t, stream, ev0);
+}
+
+// split a host/device array over the local shards ("split into portions of
+// approximately equal size"); in rank mode the whole call is this rank's portion.
+void split_io(wd_table* t, const IO& all, std::vector<IO>& ios) {
+  const size_t L = t->local.size();
+  ios.assign(L, all);
+  for (size_t r = 0; r < L; ++r) {
+    const uint64_t lo = all.n * r / L, hi = all.n * (r + 1) / L;
+    ios[r].n = hi - lo;
+    if (all.keys) ios[r].keys = all.keys + lo;
+    if (all.vals) ios[r].vals = all.vals + lo;
+    if (all.vout) ios[r].vout = all.vout + lo;
+    if (all.fout) ios[r].fout = all.fout + lo;
+  }
+}
+
+wd_status_t check_ptr(wd_table* t, const void* p, PtrKind* kind) {
+  int dev = -1;
+  *kind = classify(p, &dev);
+  if (*kind == PK_DEVICE && p) {
+    if (t->mode == MODE_MULTI)
+      return fail(WD_ERR_INVALID_ARG,
+                  "device pointers with n_gpus > 1 in one process: pass host memory");
+    if (dev != t->local[0].device)
+      return fail(WD_ERR_INVALID_ARG, "device pointer on device %d, table on device %d", dev,
+                  t->local[0].device);
+  }
+  return WD_OK;
+}
+
+wd_status_t do_op(wd_table* t, bool insert, const uint32_t* keys, const uint32_t* vals,
+                  uint32_t* vout, uint8_t* fout, uint64_t n, cudaStream_t stream) {
+  if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  if (n && !keys) return fail(WD_ERR_INVALID_ARG, "keys == NULL with n > 0");
+  if (n && insert && !vals) return fail(WD_ERR_INVALID_ARG, "vals == NULL with n > 0");
+  IO io;
+  io.keys = keys; io.vals = vals; io.vout = vout; io.fout = fout; io.n = n;
+  if (n) {
+    PtrKind k1, k2 = PK_DEVICE, k3 = PK_DEVICE;
+    TRY(check_ptr(t, keys, &k1));
+    if (insert) TRY(check_ptr(t, vals, &k2));
+    else {
+      if (vout) TRY(check_ptr(t, vout, &k2));
+      if (fout) TRY(check_ptr(t, fout, &k3));
+    }
+    if (insert && (k1 == PK_DEVICE) != (k2 == PK_DEVICE))
+      return fail(WD_ERR_INVALID_ARG, "keys and vals must both be host or both device");
+    if (!insert && vout && fout && (k2 == PK_DEVICE) != (k3 == PK_DEVICE))
+      return fail(WD_ERR_INVALID_ARG, "vals_out and found_out must both be host or device");
+    io.kin = (k1 == PK_PAGEABLE || k2 == PK_PAGEABLE) && insert ? PK_PAGEABLE : k1;
+    io.kout = insert ? PK_DEVICE : (vout ? k2 : k3);
+    if (!insert && !vout && !fout) io.kout = PK_DEVICE;
+  }
+  if (t->m == 1) {
+    if (n == 0) return WD_OK;
+    return single_op(t, insert, io, stream);
+  }
+  std::vector<IO> ios;
+  split_io(t, io, ios);
+  return cascade_op(t, insert, ios, stream);
+}
+
+wd_table* create_common(uint64_t capacity, int mode, int m, int group_size) {
+  if (capacity < 1) { fail(WD_ERR_INVALID_ARG, "capacity must be >= 1"); return nullptr; }
+  if (group_size != 1 && group_size != 2 && group_size != 4 && group_size != 8 &&
+      group_size != 16 && group_size != 32) {
+    fail(WD_ERR_INVALID_ARG, "group_size %d not in {1,2,4,8,16,32}", group_size);
+    return nullptr;
+  }
+  if (m < 1 || m > wd::kMaxShards) {
+    fail(WD_ERR_INVALID_ARG, "number of shards %d not in [1, %d]", m, wd::kMaxShards);
+    return nullptr;
+  }
+  wd_table* t = new wd_table();
+  t->mode = mode;
+  t->m = m;
+  t->G = group_size;
+  return t;
+}
+
+uint64_t shard_cap(uint64_t capacity, int m) {
+  uint64_t c = (capacity + m - 1) / m;
+  c = round_up(std::max<uint64_t>(c, 32), 4);
+  return c;
+}
+
+wd_status_t sticky_status(wd_table* t) {
+  unsigned long long agg[wd::CNT_N] = {0, 0, 0, 0};
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    unsigned long long c[wd::CNT_N];
+    CK(cudaStreamSynchronize(s.s_main));
+    CK(cudaStreamSynchronize(s.s_h2d));
+    CK(cudaStreamSynchronize(s.s_d2h));
+    CK(cudaDeviceSynchronize());
+    CK(cudaMemcpy(c, s.counters, sizeof c, cudaMemcpyDeviceToHost));
+    for (int i = 0; i < wd::CNT_N; ++i) agg[i] += c[i];
+  }
+  if (agg[wd::CNT_XERR]) return fail(WD_ERR_EXCHANGE, "%llu exchange errors (overflow/timeout)", agg[wd::CNT_XERR]);
+  if (agg[wd::CNT_FAIL]) return fail(WD_ERR_TABLE_FULL, "%llu inserts exhausted p_max", agg[wd::CNT_FAIL]);
+  if (agg[wd::CNT_RSV]) return fail(WD_ERR_RESERVED_KEY, "%llu reserved keys (0xFFFFFFFF) seen", agg[wd::CNT_RSV]);
+  return WD_OK;
+}
+
+}  // namespace
+
+// ===================================================================== C-ABI
+extern "C" {
+
+wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size) {
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) {
+    cudaGetLastError();
+    fail(WD_ERR_CUDA, "no CUDA device");
+    return nullptr;
+  }
+  if (n_gpus < 1 || n_gpus > ndev) {
+    fail(WD_ERR_INVALID_ARG, "n_gpus %d not in [1, %d visible]", n_gpus, ndev);
+    return nullptr;
+  }
+  wd_table* t = create_common(capacity, n_gpus == 1 ? MODE_SINGLE : MODE_MULTI, n_gpus, group_size);
+  if (!t) return nullptr;
+  int cur = 0;
+  cudaGetDevice(&cur);
+  cudaDeviceGetAttribute(&t->sm_count, cudaDevAttrMultiProcessorCount, n_gpus == 1 ? cur : 0);
+  const uint64_t c = shard_cap(capacity, n_gpus);
+  t->local.resize(n_gpus);
+  for (int d = 0; d < n_gpus; ++d) {
+    const int dev = n_gpus == 1 ? cur : d;
+    if (n_gpus > 1) {
+      DeviceGuard g(dev);
+      for (int p = 0; p < n_gpus; ++p)
+        if (p != dev) {
+          int ok = 0;
+          cudaDeviceCanAccessPeer(&ok, dev, p);
+          if (ok && cudaDeviceEnablePeerAccess(p, 0) != cudaSuccess) cudaGetLastError();
+        }
+    }
+    if (shard_init(t, t->local[d], d, dev, c, nullptr) != WD_OK) {
+      wd_destroy(t);
+      return nullptr;
+    }
+  }
+  g_last = WD_OK;
+  return t;
+}
+
+wd_table_t* wd_create_loopback(uint64_t capacity, int n_shards, int group_size) {
+  wd_table* t = create_common(capacity, MODE_LOOPBACK, n_shards, group_size);
+  if (!t) return nullptr;
+  int cur = 0;
+  if (cudaGetDevice(&cur) != cudaSuccess) {
+    fail(WD_ERR_CUDA, "no CUDA device");
+    delete t;
+    return nullptr;
+  }
+  cudaDeviceGetAttribute(&t->sm_count, cudaDevAttrMultiProcessorCount, cur);
+  if (cudaStreamCreateWithFlags(&t->loop_stream, cudaStreamNonBlocking) != cudaSuccess) {
+    fail(WD_ERR_CUDA, "stream creation failed");
+    delete t;
+    return nullptr;
+  }
+  const uint64_t c = shard_cap(capacity, n_shards);
+  t->local.resize(n_shards);
+  for (int d = 0; d < n_shards; ++d)
+    if (shard_init(t, t->local[d], d, cur, c, t->loop_stream) != WD_OK) {
+      wd_destroy(t);
+      return nullptr;
+    }
+  g_last = WD_OK;
+  return t;
+}
+
+wd_status_t wd_get_unique_id(uint8_t unique_id[128]) {
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+  ncclUniqueId id;
+  NK(ncclGetUniqueId(&id));
+  memcpy(unique_id, &id, 128);
+  return WD_OK;
+}
+
+wd_table_t* wd_create_rank(uint64_t capacity, int rank, int world, const uint8_t unique_id[128],
+                           int group_size) {
+  if (world < 1 || rank < 0 || rank >= world || !unique_id) {
+    fail(WD_ERR_INVALID_ARG, "rank %d / world %d", rank, world);
+    return nullptr;
+  }
+  wd_table* t = create_common(capacity, world == 1 ? MODE_SINGLE : MODE_RANK, world, group_size);
+  if (!t) return nullptr;
+  t->rank = rank;
+  int cur = 0;
+  if (cudaGetDevice(&cur) != cudaSuccess) {
+    fail(WD_ERR_CUDA, "no CUDA device");
+    delete t;
+    return nullptr;
+  }
+  cudaDeviceGetAttribute(&t->sm_count, cudaDevAttrMultiProcessorCount, cur);
+  t->local.resize(1);
+  if (shard_init(t, t->local[0], rank, cur, shard_cap(capacity, world), nullptr) != WD_OK) {
+    wd_destroy(t);
+    return nullptr;
+  }
+  if (world > 1) {
+    ncclUniqueId id;
+    memcpy(&id, unique_id, 128);
+    ncclResult_t r = ncclCommInitRank(&t->comm, world, id, rank);
+    if (r != ncclSuccess) {
+      fail(WD_ERR_NCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+      wd_destroy(t);
+      return nullptr;
+    }
+    if (cudaMalloc(&t->d_scratch, 64) != cudaSuccess || ensure_exchange(t) != WD_OK) {
+      if (g_last == WD_OK) fail(WD_ERR_OUT_OF_MEMORY, "scratch allocation");
+      wd_destroy(t);
+      return nullptr;
+    }
+  }
+  g_last = WD_OK;
+  return t;
+}
+
+void wd_destroy(wd_table_t* t) {
+  if (!t) return;
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    cudaDeviceSynchronize();
+  }
+  if (t->comm) {  // collective: no rank unmaps before every rank is done
+    ncclAllReduce(t->d_scratch, t->d_scratch, 1, ncclUint64, ncclSum, t->comm,
+                  t->local[0].s_main);
+    cudaStreamSynchronize(t->local[0].s_main);
+  }
+  for (void* p : t->opened) cudaIpcCloseMemHandle(p);
+  for (auto& s : t->local) shard_free(s);
+  if (t->comm) ncclCommDestroy(t->comm);
+  if (t->d_scratch) cudaFree(t->d_scratch);
+  if (t->loop_stream) cudaStreamDestroy(t->loop_stream);
+  delete t;
+}
+
+wd_status_t wd_clear(wd_table_t* t, wd_stream_t stream) {
+  if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  if (t->mode == MODE_SINGLE) {
+    Shard& s = t->local[0];
+    DeviceGuard g(s.device);
+    wd::fill_kernel<<<t->sm_count * 4, wd::kBlock, 0, st>>>(s.slots, s.cap, s.counters, wd::CNT_N);
+    CK(cudaGetLastError());
+    t->launches++;
+    return WD_OK;
+  }
+  cudaEvent_t ev0;
+  TRY(fork_from(t, st, &ev0));
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    wd::fill_kernel<<<t->sm_count * 4, wd::kBlock, 0, s.s_main>>>(s.slots, s.cap, s.counters,
+                                                                  wd::CNT_N);
+    CK(cudaGetLastError());
+    t->launches++;
+  }
+  return join_into(t, st, ev0);
+}
+
+wd_status_t wd_insert(wd_table_t* t, const uint32_t* keys, const uint32_t* vals, uint64_t n,
+                      wd_stream_t stream) {
+  return do_op(t, true, keys, vals, nullptr, nullptr, n, reinterpret_cast<cudaStream_t>(stream));
+}
+
+wd_status_t wd_retrieve(wd_table_t* t, const uint32_t* keys, uint32_t* vals_out, uint8_t* found_out,
+                        uint64_t n, wd_stream_t stream) {
+  return do_op(t, false, keys, nullptr, vals_out, found_out, n,
+               reinterpret_cast<cudaStream_t>(stream));
+}
+
+wd_status_t wd_sync(wd_table_t* t) {
+  if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  return sticky_status(t);
+}
+
+uint64_t wd_size(wd_table_t* t) {
+  if (!t) { fail(WD_ERR_INVALID_ARG, "null table"); return UINT64_MAX; }
+  unsigned long long total = 0;
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    unsigned long long c = 0;
+    if (cudaDeviceSynchronize() != cudaSuccess ||
+        cudaMemcpy(&c, s.counters + wd::CNT_NEW, 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+      fail(WD_ERR_CUDA, "wd_size: %s", cudaGetErrorString(cudaGetLastError()));
+      return UINT64_MAX;
+    }
+    total += c;
+  }
+  if (t->mode == MODE_RANK) {
+    Shard& s = t->local[0];
+    DeviceGuard g(s.device);
+    if (cudaMemcpy(t->d_scratch, &total, 8, cudaMemcpyHostToDevice) != cudaSuccess ||
+        ncclAllReduce(t->d_scratch, t->d_scratch, 1, ncclUint64, ncclSum, t->comm, s.s_main) !=
+            ncclSuccess ||
+        cudaStreamSynchronize(s.s_main) != cudaSuccess ||
+        cudaMemcpy(&total, t->d_scratch, 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+      fail(WD_ERR_NCCL, "wd_size allreduce failed");
+      return UINT64_MAX;
+    }
+  }
+  return total;
+}
+
+uint64_t wd_capacity(wd_table_t* t) {
+  if (!t) return 0;
+  return t->local[0].cap * uint64_t(t->m);
+}
+
+wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
+  if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  switch (opt) {
+    case WD_OPT_GROUP_SIZE:
+      if (v != 1 && v != 2 && v != 4 && v != 8 && v != 16 && v != 32)
+        return fail(WD_ERR_INVALID_ARG, "group size %lld", (long long)v);
+      t->G = int(v);
+      return WD_OK;
+    case WD_OPT_P_MAX:
+      if (v < 1 || v > (1 << 20)) return fail(WD_ERR_INVALID_ARG, "p_max %lld", (long long)v);
+      t->pmax = int(v);
+      return WD_OK;
+    case WD_OPT_BATCH:
+      if (v < 1 || v > (1ll << wd::kPosShift)) return fail(WD_ERR_INVALID_ARG, "batch %lld", (long long)v);
+      t->batch = uint64_t(v);
+      return WD_OK;
+    case WD_OPT_SERIAL: t->serial = v ? 1 : 0; return WD_OK;
+    case WD_OPT_KEYS_IN_FLIGHT:
+      if (v != 0 && v != 4 && v != 8) return fail(WD_ERR_INVALID_ARG, "keys in flight %lld", (long long)v);
+      t->kif = int(v);
+      return WD_OK;
+    case WD_OPT_PART_SEED: t->pseed = uint32_t(v); return WD_OK;
+    case WD_OPT_PART_MODE:
+      if (v != 0 && v != 1) return fail(WD_ERR_INVALID_ARG, "partition mode %lld", (long long)v);
+      t->pmode = int(v);
+      return WD_OK;
+    default: return fail(WD_ERR_INVALID_ARG, "option %d is read-only or unknown", int(opt));
+  }
+}
+
+int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
+  if (!t) { fail(WD_ERR_INVALID_ARG, "null table"); return INT64_MIN; }
+  switch (opt) {
+    case WD_OPT_GROUP_SIZE: return t->G;
+    case WD_OPT_P_MAX: return t->pmax;
+    case WD_OPT_BATCH: return int64_t(t->batch);
+    case WD_OPT_SERIAL: return t->serial;
+    case WD_OPT_KEYS_IN_FLIGHT: return t->kif ? t->kif : (t->G <= 2 ? 4 : 8);
+    case WD_OPT_PART_SEED: return t->pseed;
+    case WD_OPT_PART_MODE: return t->pmode;
+    case WD_OPT_N_SHARDS: return t->m;
+    case WD_OPT_RANK: return t->rank;
+    case WD_OPT_LOCAL_SHARDS: return int64_t(t->local.size());
+    case WD_OPT_LAUNCHES: return int64_t(t->launches);
+  }
+  fail(WD_ERR_INVALID_ARG, "unknown option %d", int(opt));
+  return INT64_MIN;
+}
+
+wd_status_t wd_last_error(void) { return g_last; }
+
+const char* wd_error_string(wd_status_t s) {
+  switch (s) {
+    case WD_OK: return "WD_OK";
+    case WD_ERR_INVALID_ARG: return "WD_ERR_INVALID_ARG";
+    case WD_ERR_OUT_OF_MEMORY: return "WD_ERR_OUT_OF_MEMORY";
+    case WD_ERR_CUDA: return "WD_ERR_CUDA";
+    case WD_ERR_NCCL: return "WD_ERR_NCCL";
+    case WD_ERR_TABLE_FULL: return "WD_ERR_TABLE_FULL";
+    case WD_ERR_RESERVED_KEY: return "WD_ERR_RESERVED_KEY";
+    case WD_ERR_EXCHANGE: return "WD_ERR_EXCHANGE";
+    case WD_ERR_UNSUPPORTED: return "WD_ERR_UNSUPPORTED";
+  }
+  return "WD_ERR_UNKNOWN";
+}
+
+const char* wd_last_error_message(void) { return g_msg; }
+
+uint64_t wd_shard_capacity(wd_table_t* t, int shard) {
+  if (!t || shard < 0 || shard >= int(t->local.size())) return 0;
+  return t->local[shard].cap;
+}
+
+wd_status_t wd_dump(wd_table_t* t, int shard, uint64_t* host_out) {
+  if (!t || shard < 0 || shard >= int(t->local.size()) || !host_out)
+    return fail(WD_ERR_INVALID_ARG, "wd_dump arguments");
+  Shard& s = t->local[shard];
+  DeviceGuard g(s.device);
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(host_out, s.slots, s.cap * 8, cudaMemcpyDeviceToHost));
+  return WD_OK;
+}
+
+wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[4]) {
+  if (!t || shard < 0 || shard >= int(t->local.size()) || !out)
+    return fail(WD_ERR_INVALID_ARG, "wd_counters arguments");
+  Shard& s = t->local[shard];
+  DeviceGuard g(s.device);
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(out, s.counters, 4 * 8, cudaMemcpyDeviceToHost));
+  return WD_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,34 @@
+"""The device-side generator equals the numpy generator element by element."""
+import numpy as np
+import pytest
+
+import wdgen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def gg():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import wdgen.gpu as gg
+    return gg
+
+
+def _np(t):
+    return t.cpu().numpy().view(np.uint32)
+
+
+def test_streams_match(gg):
+    n, start = 300_017, 123_456
+    assert np.array_equal(_np(gg.unique_keys(n, 5, start)), wdgen.unique_keys(n, 5, start))
+    assert np.array_equal(_np(gg.values(n, 6, start)), wdgen.values(n, 6, start))
+    assert np.array_equal(_np(gg.uniform_keys(n, 7, start)), wdgen.uniform_keys(n, 7, start))
+    assert np.array_equal(_np(gg.interleaved_queries(1000, 8, 10, 1990)),
+                          wdgen.interleaved_queries(1000, 8, 10, 1990))
+    import torch
+    hits = torch.empty(n, dtype=torch.uint8, device="cuda")
+    q = gg.mixed_queries(50_000, n, 0.5, 9, start, hits=hits)
+    eq, eh = wdgen.mixed_queries(50_000, n, 0.5, 9, start)
+    assert np.array_equal(_np(q), eq) and np.array_equal(hits.cpu().numpy().astype(bool), eh)

@@ -1,0 +1,93 @@
+"""Multi-shard cascade on ONE GPU: m virtual shards (wd_create_loopback) run the full
+multi-GPU path — multisplit fused with the push into the owners' receive regions,
+T row/column via flags, local insert/query, reverse pull + unpermute — with peer pointers
+that happen to be local.  Results must equal the oracle bit for bit (the paper's
+"transparent scaling", P:7), and every shard must hold exactly its partition."""
+import numpy as np
+import pytest
+
+import oracle
+import wdgen
+from wdtest import capacity_for, from_dev, gpu_roundtrip, to_dev
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def wd():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_ipps_junger0s18_b200 as wd
+    return wd
+
+
+@pytest.mark.parametrize("m", [2, 3, 4, 8])
+@pytest.mark.parametrize("G", [1, 4, 32])
+def test_loopback_unique_parity(wd, m, G):
+    n = 200_000 + 17 * m
+    keys, vals = wdgen.unique_keys(n, 21), wdgen.values(n, 22)
+    q = wdgen.interleaved_queries(n, 21)
+    with wd.Table(capacity_for(n, 0.9), group_size=G, loopback_shards=m) as t:
+        t.set_option(wd.WD_OPT_BATCH, 9_000)  # many batches per shard: epochs wrap slots
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0, wd._lib.wd_last_error_message()
+        assert t.size() == n
+        seed = t.get_option(wd.WD_OPT_PART_SEED)
+        # shard d holds exactly the keys with p(k) = d
+        for d in range(m):
+            sl = t.dump(d)
+            k = (sl & np.uint64(0xFFFFFFFF)).astype(np.uint32)
+            k = k[k != np.uint32(0xFFFFFFFF)]
+            assert np.all(oracle.partition(k, m, seed) == d)
+            assert t.counters(d)["exchange_errors"] == 0
+    cv, cf = oracle.expected_unique(q, n, 21, 22)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
+@pytest.mark.parametrize("m", [2, 4])
+def test_loopback_host_and_dups(wd, m):
+    n = 120_000
+    keys = wdgen.uniform_keys(n, 31) % np.uint32(50_000)
+    vals = wdgen.values(n, 32)
+    q = np.arange(60_000, dtype=np.uint32)
+    with wd.Table(capacity_for(50_000, 0.85), group_size=4, loopback_shards=m) as t:
+        t.set_option(wd.WD_OPT_BATCH, 5_000)
+        gv, gf = gpu_roundtrip(t, keys, vals, q, host=True)
+        assert t.sync() == 0
+        mo = oracle.Map(n, dup_mode=True)
+        mo.insert(keys, vals)
+        assert t.size() == mo.size()
+    ev, ef = mo.retrieve(q)
+    assert np.array_equal(gf, ef)
+    assert np.all(mo.pair_status(q[gf == 1], gv[gf == 1]) >= 1)
+
+
+def test_loopback_fig4_partition_mode(wd):
+    # Fig. 4: p(k) = k mod 4 over 4 shards
+    keys = np.arange(1, 4001, dtype=np.uint32) * 3
+    vals = keys ^ np.uint32(0xABCDEF)
+    with wd.Table(6000, group_size=2, loopback_shards=4) as t:
+        t.set_option(wd.WD_OPT_PART_MODE, 1)
+        t.set_option(wd.WD_OPT_BATCH, 333)
+        gv, gf = gpu_roundtrip(t, keys, vals, np.concatenate([keys, keys + 1]))
+        for d in range(4):
+            sl = t.dump(d)
+            k = (sl & np.uint64(0xFFFFFFFF)).astype(np.uint32)
+            k = k[k != np.uint32(0xFFFFFFFF)]
+            assert np.all(k % 4 == d)
+        assert t.size() == keys.size
+    assert np.all(gf[:4000] == 1) and np.array_equal(gv[:4000], vals)
+    kk = keys + 1
+    present = np.isin(kk, keys)
+    assert np.array_equal(gf[4000:].astype(bool), present)
+
+
+def test_loopback_uneven_and_empty(wd):
+    # one call with fewer items than shards, then n = 0
+    with wd.Table(1000, group_size=4, loopback_shards=8) as t:
+        gv, gf = gpu_roundtrip(t, np.array([5, 6, 7], np.uint32), np.array([1, 2, 3], np.uint32),
+                               np.array([7, 6, 5, 4], np.uint32))
+        assert list(gf) == [1, 1, 1, 0] and list(gv[:3]) == [3, 2, 1]
+        t.insert(to_dev(np.zeros(0, np.uint32)), to_dev(np.zeros(0, np.uint32)))
+        assert t.sync() == 0 and t.size() == 3

@@ -1,0 +1,214 @@
+"""Single-GPU parity: the CUDA path (through the C-ABI) against the oracle, element by
+element, bit-exact on (found, value).  Marked gpu: run on the B200 box."""
+import numpy as np
+import pytest
+
+import oracle
+import wdgen
+from wdtest import capacity_for, from_dev, gpu_roundtrip, to_dev
+
+pytestmark = pytest.mark.gpu
+
+GS = [1, 2, 4, 8, 16, 32]
+
+
+@pytest.fixture(scope="module")
+def wd():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_ipps_junger0s18_b200 as wd
+    return wd
+
+
+def _oracle_answers(keys, vals, queries, dup=False):
+    m = oracle.Map(keys.size, dup_mode=dup)
+    m.insert(keys, vals)
+    return m, *m.retrieve(queries)
+
+
+@pytest.mark.parametrize("G", GS)
+def test_config1_unique_parity(wd, G):
+    # BASELINE config 1: 2^20 unique keys, load 0.95, all keys + 2^20 absent keys queried
+    n, ks, vs = 1 << 20, 101, 202
+    keys, vals = wdgen.unique_keys(n, ks), wdgen.values(n, vs)
+    q = wdgen.interleaved_queries(n, ks)
+    with wd.Table(capacity_for(n, 0.95), 1, G) as t:
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0
+        assert t.size() == n
+        cnt = t.counters()
+        assert cnt["failed"] == 0 and cnt["reserved"] == 0
+        load = t.size() / t.capacity()
+        assert abs(load - 0.95) < 1e-3
+    m, ev, ef = _oracle_answers(keys, vals, q)
+    assert np.array_equal(gf, ef)
+    assert np.array_equal(gv, ev)
+    # closed form (independent of the oracle's table)
+    cv, cf = oracle.expected_unique(q, n, ks, vs)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
+@pytest.mark.parametrize("kif", [4, 8])
+@pytest.mark.parametrize("alpha", [0.8, 0.99])
+def test_alpha_and_keys_in_flight(wd, alpha, kif):
+    n = 300_001  # ragged
+    keys, vals = wdgen.unique_keys(n, 7), wdgen.values(n, 8)
+    q = wdgen.interleaved_queries(n, 7)
+    with wd.Table(capacity_for(n, alpha), 1, 4) as t:
+        t.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, kif)
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0 and t.size() == n
+    cv, cf = oracle.expected_unique(q, n, 7, 8)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
+@pytest.mark.parametrize("G", GS)
+def test_serial_layout_equals_fig3_replay(wd, G):
+    # WD_OPT_SERIAL runs one probing group, one key at a time: the slot layout must equal
+    # the oracle's sequential replay of Fig. 3 bit for bit (probe sequence, windows,
+    # leftmost-empty leader, update-on-match).
+    n = 3000
+    c = 3200
+    keys = np.concatenate([wdgen.unique_keys(n, 3), wdgen.unique_keys(200, 3)])  # 200 updates
+    vals = wdgen.values(n + 200, 4)
+    r = oracle.Replay(c, G)
+    r.insert(keys, vals)
+    with wd.Table(c, 1, G) as t:
+        t.set_option(wd.WD_OPT_SERIAL, 1)
+        t.insert(to_dev(keys), to_dev(vals))
+        assert t.sync() == 0
+        slots = t.dump()
+        assert t.size() == n
+    assert np.array_equal(slots, r.table)
+
+
+@pytest.mark.parametrize("Gi,Gq", [(1, 32), (32, 1), (4, 8), (8, 2), (2, 16)])
+def test_cross_group_size(wd, Gi, Gq):
+    # the probing scheme is consistent when |g| varies: insert with one |g|, query
+    # with another.
+    n = 200_000
+    keys, vals = wdgen.unique_keys(n, 9), wdgen.values(n, 9)
+    q = wdgen.interleaved_queries(n, 9)
+    with wd.Table(capacity_for(n, 0.97), 1, Gi) as t:
+        t.insert(to_dev(keys), to_dev(vals))
+        t.set_option(wd.WD_OPT_GROUP_SIZE, Gq)
+        ov, of = t.retrieve(to_dev(q))
+        gv, gf = from_dev(ov), of.cpu().numpy()
+    cv, cf = oracle.expected_unique(q, n, 9, 9)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
+@pytest.mark.parametrize("G", [1, 4, 32])
+def test_duplicates_upsert(wd, G):
+    # duplicate-key mode: value must be one of the values inserted for the key;
+    # size = number of distinct keys; a second stream-ordered call wins.
+    n = 400_000
+    keys = wdgen.uniform_keys(n, 11) % np.uint32(150_000)
+    vals = wdgen.values(n, 12)
+    with wd.Table(capacity_for(150_000, 0.9), 1, G) as t:
+        t.insert(to_dev(keys), to_dev(vals))
+        q = np.arange(160_000, dtype=np.uint32)
+        ov, of = t.retrieve(to_dev(q))
+        gv, gf = from_dev(ov), of.cpu().numpy()
+        m = oracle.Map(n, dup_mode=True)
+        m.insert(keys, vals)
+        assert t.size() == m.size()
+        ev, ef = m.retrieve(q)
+        assert np.array_equal(gf, ef)
+        st = m.pair_status(q[gf == 1], gv[gf == 1])
+        assert np.all(st >= 1)          # v in V(k)
+        assert np.all(gv[gf == 0] == 0xFFFFFFFF)
+        # second call overwrites: last call wins
+        k2 = np.unique(keys)[:1000]
+        v2 = wdgen.values(k2.size, 99)
+        t.insert(to_dev(k2), to_dev(v2))
+        ov, of = t.retrieve(to_dev(k2))
+        assert np.array_equal(from_dev(ov), v2)
+        assert t.size() == m.size()
+
+
+def test_edge_cases(wd):
+    import torch
+    # exactly full: c = 32 (one region), 32 keys, alpha = 1
+    keys, vals = wdgen.unique_keys(33, 5), wdgen.values(33, 5)
+    with wd.Table(32, 1, 4) as t:
+        assert t.capacity() == 32
+        gv, gf = gpu_roundtrip(t, keys[:32], vals[:32], keys)
+        assert t.sync() == 0 and t.size() == 32
+        assert np.all(gf[:32] == 1) and np.array_equal(gv[:32], vals[:32]) and gf[32] == 0
+        # alpha > 1: the 33rd key cannot be placed
+        t.set_option(wd.WD_OPT_P_MAX, 4)
+        t.insert(to_dev(keys[32:]), to_dev(vals[32:]))
+        assert t.sync() == wd.WD_ERR_TABLE_FULL
+        assert t.counters()["failed"] == 1 and t.size() == 32
+        t.clear()
+        torch.cuda.synchronize()
+        assert t.sync() == 0 and t.size() == 0
+    # reserved key and 0xFFFFFFFF values
+    keys = np.array([1, 0xFFFFFFFF, 2, 0, 3], np.uint32)
+    vals = np.array([0xFFFFFFFF, 7, 0, 0xFFFFFFFF, 5], np.uint32)
+    q = np.array([0, 1, 2, 3, 0xFFFFFFFF, 4], np.uint32)
+    with wd.Table(64, 1, 8) as t:
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == wd.WD_ERR_RESERVED_KEY
+        assert t.size() == 4
+        m, ev, ef = _oracle_answers(keys, vals, q)
+        assert np.array_equal(gf, ef) and np.array_equal(gv, ev)
+    # n = 0 and n = 1
+    with wd.Table(100, 1, 4) as t:
+        t.insert(to_dev(np.zeros(0, np.uint32)), to_dev(np.zeros(0, np.uint32)))
+        ov, of = t.retrieve(to_dev(np.zeros(0, np.uint32)))
+        assert ov.numel() == 0
+        gv, gf = gpu_roundtrip(t, np.array([42], np.uint32), np.array([43], np.uint32),
+                               np.array([42, 41], np.uint32))
+        assert list(gf) == [1, 0] and gv[0] == 43 and gv[1] == 0xFFFFFFFF
+    # bad arguments
+    with pytest.raises(wd.WarpDriveError):
+        wd.Table(100, 1, 3)
+    with pytest.raises(wd.WarpDriveError):
+        wd.Table(0, 1, 4)
+
+
+@pytest.mark.parametrize("pinned", [True, False])
+def test_host_pointers_out_of_core(wd, pinned):
+    # a11: host-resident input streamed in batches; tiny batch -> many batches
+    n = 100_003
+    keys, vals = wdgen.unique_keys(n, 13), wdgen.values(n, 14)
+    q = wdgen.interleaved_queries(n, 13)
+    with wd.Table(capacity_for(n, 0.95), 1, 4) as t:
+        t.set_option(wd.WD_OPT_BATCH, 7_777)
+        if pinned:
+            gv, gf = gpu_roundtrip(t, keys, vals, q, host=True)
+        else:
+            t.insert(keys, vals)           # numpy (pageable)
+            gv, gf = t.retrieve(q)
+        assert t.sync() == 0 and t.size() == n
+    cv, cf = oracle.expected_unique(q, n, 13, 14)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
+def test_config2_full_size_sampled(wd):
+    # BASELINE config 2 at its full size (2^28 unique pairs, alpha 0.95, |g| = 4), inputs
+    # generated on the device; every query checked in-kernel-order against the closed
+    # form on a 2^22 sample of positions spanning the whole range.
+    import torch
+    import wdgen.gpu as gg
+    n, ks, vs = 1 << 28, 77, 78
+    keys, vals = gg.unique_keys(n, ks), gg.values(n, vs)
+    with wd.Table(capacity_for(n, 0.95), 1, 4) as t:
+        t.insert(keys, vals)
+        del vals
+        q = gg.interleaved_queries(n, ks, start=n - (1 << 27), count=1 << 28)  # half present
+        ov, of = t.retrieve(q)
+        assert t.sync() == 0 and t.size() == n
+        torch.cuda.synchronize()
+        rng = np.random.default_rng(0)
+        idx = np.sort(rng.choice(q.numel(), 1 << 22, replace=False))
+        ii = torch.from_numpy(idx).cuda()
+        qs = q[ii].cpu().numpy().view(np.uint32)
+        gv = ov[ii].cpu().numpy().view(np.uint32)
+        gf = of[ii].cpu().numpy()
+    cv, cf = oracle.expected_unique(qs, n, ks, vs)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+    assert 0.45 < gf.mean() < 0.55

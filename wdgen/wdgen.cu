@@ -1,0 +1,116 @@
+// wdgen.cu — device-side copy of the counter-based input generator of wdgen/__init__.py.
+// Generator only (no hashing/probing/partitioning of the method): used by the bench and
+// the large GPU tests to create inputs in HBM without a host round trip; never timed
+// ("test data generation ... omitted").  tests/test_gen_gpu.py checks it equals
+// the numpy version element by element.
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace {
+constexpr uint32_t kEmpty = 0xFFFFFFFFu;
+constexpr uint64_t TAG_PERM = 0x5045524D, TAG_VAL = 0x56414C55, TAG_UNI = 0x554E4946,
+                   TAG_MIX = 0x4D495851;
+
+__host__ __device__ inline uint64_t splitmix64(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+__host__ __device__ inline uint64_t stream_key(uint64_t seed, uint64_t tag) {
+  return splitmix64(seed ^ (tag << 32));
+}
+struct RK { uint64_t k[4]; };
+RK round_keys(uint64_t seed) {
+  RK r;
+  const uint64_t base = stream_key(seed, TAG_PERM);
+  for (int i = 0; i < 4; ++i) r.k[i] = splitmix64(base + i);
+  return r;
+}
+__device__ inline uint32_t feistel(uint32_t x, const RK& rk) {
+  uint64_t L = x >> 16, R = x & 0xFFFF;
+#pragma unroll
+  for (int r = 0; r < 4; ++r) {
+    const uint64_t F = splitmix64(R ^ rk.k[r]) & 0xFFFF;
+    const uint64_t nl = R;
+    R = L ^ F;
+    L = nl;
+  }
+  return uint32_t((L << 16) | R);
+}
+__device__ inline uint32_t perm32(uint32_t x, const RK& rk) {
+  uint32_t y = feistel(x, rk);
+  if (y == kEmpty) y = feistel(kEmpty, rk);
+  return y;
+}
+
+__global__ void k_unique(uint32_t* out, uint64_t start, uint64_t n, RK rk) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x)
+    out[i] = perm32(uint32_t(start + i), rk);
+}
+__global__ void k_values(uint32_t* out, uint64_t start, uint64_t n, uint64_t sk) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x)
+    out[i] = uint32_t(splitmix64(start + i + sk));
+}
+__global__ void k_uniform(uint32_t* out, uint64_t start, uint64_t n, uint64_t sk) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t z = splitmix64(start + i + sk);
+    uint32_t k = uint32_t(z);
+    if (k == kEmpty) k = uint32_t(z >> 32);
+    if (k == kEmpty) k = 0;
+    out[i] = k;
+  }
+}
+__global__ void k_interleaved(uint32_t* out, uint64_t n_present, uint64_t start, uint64_t count, RK rk) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < count; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t j = start + i;
+    const uint64_t idx = (j >> 1) + (j & 1) * n_present;
+    out[i] = perm32(uint32_t(idx), rk);
+  }
+}
+__global__ void k_mixed(uint32_t* out, uint8_t* hit_out, uint64_t n_table, uint64_t start, uint64_t count,
+                        uint64_t thr, uint64_t sk, RK rk) {
+  const uint64_t n_abs = uint64_t(kEmpty) - n_table;
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < count; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t z = splitmix64(start + i + sk);
+    const uint64_t lo = z & 0xFFFFFFFFull, r = z >> 32;
+    const bool hit = lo < thr;
+    const uint64_t idx = hit ? r % (n_table ? n_table : 1) : n_table + r % n_abs;
+    out[i] = perm32(uint32_t(idx), rk);
+    if (hit_out) hit_out[i] = hit;
+  }
+}
+int grid_for(uint64_t n) {
+  uint64_t g = (n + 255) / 256;
+  return int(g < 148 * 16 ? (g ? g : 1) : 148 * 16);
+}
+}  // namespace
+
+extern "C" {
+int wdgen_unique_keys(uint32_t* out, uint64_t start, uint64_t n, uint64_t seed, cudaStream_t st) {
+  if (n) k_unique<<<grid_for(n), 256, 0, st>>>(out, start, n, round_keys(seed));
+  return int(cudaGetLastError());
+}
+int wdgen_values(uint32_t* out, uint64_t start, uint64_t n, uint64_t seed, cudaStream_t st) {
+  if (n) k_values<<<grid_for(n), 256, 0, st>>>(out, start, n, stream_key(seed, TAG_VAL));
+  return int(cudaGetLastError());
+}
+int wdgen_uniform_keys(uint32_t* out, uint64_t start, uint64_t n, uint64_t seed, cudaStream_t st) {
+  if (n) k_uniform<<<grid_for(n), 256, 0, st>>>(out, start, n, stream_key(seed, TAG_UNI));
+  return int(cudaGetLastError());
+}
+int wdgen_interleaved_queries(uint32_t* out, uint64_t n_present, uint64_t start, uint64_t count,
+                              uint64_t seed, cudaStream_t st) {
+  if (count) k_interleaved<<<grid_for(count), 256, 0, st>>>(out, n_present, start, count, round_keys(seed));
+  return int(cudaGetLastError());
+}
+int wdgen_mixed_queries(uint32_t* out, uint8_t* hit_out, uint64_t n_table, uint64_t start, uint64_t count,
+                        double hit_frac, uint64_t seed, cudaStream_t st) {
+  double t = hit_frac * 4294967296.0;
+  uint64_t thr = t >= 4294967296.0 ? 4294967296ull : (t <= 0 ? 0ull : uint64_t(t));
+  if (count)
+    k_mixed<<<grid_for(count), 256, 0, st>>>(out, hit_out, n_table, start, count, thr,
+                                             stream_key(seed, TAG_MIX), round_keys(seed));
+  return int(cudaGetLastError());
+}
+}
