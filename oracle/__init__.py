@@ -75,6 +75,7 @@ def lib():
         L.or_replay_query.argtypes = [p, u64, C.c_int, u32, p, p, p, u64, C.POINTER(_Stats)]
         L.or_replay_query.restype = None
         L.or_replay_base.argtypes = [u32, u32, u64]; L.or_replay_base.restype = u64
+        L.or_physical_capacity.argtypes = [u64]; L.or_physical_capacity.restype = u64
         for f in (L.or_fmix32_many, L.or_mueller_many):
             f.argtypes = [p, p, u64]; f.restype = None
         L.or_partition_many.argtypes = [p, p, u64, u32, u32, C.c_int]
@@ -211,6 +212,12 @@ class Replay:
     @staticmethod
     def base(k: int, p: int, capacity: int) -> int:
         return int(lib().or_replay_base(int(k), int(p), int(capacity)))
+
+
+def physical_capacity(c: int) -> int:
+    """Slots a table of requested capacity c must have so that eq. 3 has full period
+    (nb = (c-32)/4 + 1 prime; reading C13')."""
+    return int(lib().or_physical_capacity(int(c)))
 
 
 # ---------------------------------------------------------------- closed form (generator)

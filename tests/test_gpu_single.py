@@ -39,6 +39,7 @@ def test_config1_unique_parity(wd, G):
         assert t.size() == n
         cnt = t.counters()
         assert cnt["failed"] == 0 and cnt["reserved"] == 0
+        assert t.capacity() == oracle.physical_capacity(capacity_for(n, 0.95))
         load = t.size() / t.capacity()
         assert abs(load - 0.95) < 1e-3
     m, ev, ef = _oracle_answers(keys, vals, q)
@@ -50,7 +51,7 @@ def test_config1_unique_parity(wd, G):
 
 
 @pytest.mark.parametrize("kif", [4, 8])
-@pytest.mark.parametrize("alpha", [0.8, 0.99])
+@pytest.mark.parametrize("alpha", [0.8, 0.99, 0.999])
 def test_alpha_and_keys_in_flight(wd, alpha, kif):
     n = 300_001  # ragged
     keys, vals = wdgen.unique_keys(n, 7), wdgen.values(n, 8)
@@ -69,12 +70,13 @@ def test_serial_layout_equals_fig3_replay(wd, G):
     # the oracle's sequential replay of Fig. 3 bit for bit (probe sequence, windows,
     # leftmost-empty leader, update-on-match).
     n = 3000
-    c = 3200
+    c = oracle.physical_capacity(3200)
     keys = np.concatenate([wdgen.unique_keys(n, 3), wdgen.unique_keys(200, 3)])  # 200 updates
     vals = wdgen.values(n + 200, 4)
     r = oracle.Replay(c, G)
     r.insert(keys, vals)
-    with wd.Table(c, 1, G) as t:
+    with wd.Table(3200, 1, G) as t:
+        assert t.shard_capacity() == c
         t.set_option(wd.WD_OPT_SERIAL, 1)
         t.insert(to_dev(keys), to_dev(vals))
         assert t.sync() == 0
@@ -145,6 +147,15 @@ def test_edge_cases(wd):
         t.clear()
         torch.cuda.synchronize()
         assert t.sync() == 0 and t.size() == 0
+    # alpha = 1 on a multi-region table: p_max >= nb reaches every slot
+    c = oracle.physical_capacity(1000)
+    keys = wdgen.unique_keys(c, 6)
+    with wd.Table(1000, 1, 4) as t:
+        assert t.capacity() == c
+        t.set_option(wd.WD_OPT_P_MAX, (c - 32) // 4 + 1)
+        gv, gf = gpu_roundtrip(t, keys, keys ^ np.uint32(1), keys)
+        assert t.sync() == 0 and t.size() == c and np.all(gf == 1)
+        assert np.array_equal(gv, keys ^ np.uint32(1))
     # reserved key and 0xFFFFFFFF values
     keys = np.array([1, 0xFFFFFFFF, 2, 0, 3], np.uint32)
     vals = np.array([0xFFFFFFFF, 7, 0, 0xFFFFFFFF, 5], np.uint32)

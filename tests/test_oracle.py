@@ -274,6 +274,55 @@ def test_replay_base_range():
     assert hist.min() >= 1 and hist.max() < 5 * hist.mean()
 
 
+def _isprime(x):
+    if x < 2:
+        return False
+    d = 2
+    while d * d <= x:
+        if x % d == 0:
+            return False
+        d += 1
+    return True
+
+
+def test_physical_capacity_prime_region_count():
+    # C13': c rounded up (multiple of 4, >= 32) until nb = (c-32)/4 + 1 is prime; minimal
+    for c in [1, 31, 32, 33, 36, 40, 64, 100, 1000, 3200, 6321, 1103765, 282563638]:
+        cp = oracle.physical_capacity(c)
+        assert cp >= max(c, 32) and cp % 4 == 0
+        nb = (cp - 32) // 4 + 1
+        assert nb == 1 or _isprime(nb)
+        c4 = max(32, (c + 3) // 4 * 4)
+        for smaller in range(c4, cp, 4):          # no smaller valid capacity
+            nbs = (smaller - 32) // 4 + 1
+            assert not (nbs == 1 or _isprime(nbs))
+
+
+@pytest.mark.parametrize("nb", [2, 3, 13, 101, 1009])
+def test_replay_region_sequence_full_period(nb):
+    # eq. 3 with a prime number of region starts and a step in [1, nb-1] visits every
+    # region exactly once in nb steps, for every key (Knuth's double-hashing condition).
+    c = 4 * (nb - 1) + 32
+    for k in wdgen.unique_keys(50, nb):
+        seq = [oracle.Replay.base(int(k), p, c) // 4 for p in range(nb)]
+        assert sorted(seq) == list(range(nb))
+        assert oracle.Replay.base(int(k), nb, c) == seq[0] * 4   # then it repeats
+
+
+@pytest.mark.parametrize("G", [1, 4, 32])
+def test_replay_fills_table_completely(G):
+    # with p_max >= nb every slot is reachable: a table can be filled to alpha = 1
+    c = oracle.physical_capacity(400)
+    nb = (c - 32) // 4 + 1
+    r = oracle.Replay(c, G, p_max=nb)
+    keys = wdgen.unique_keys(c + 1, 17)
+    r.insert(keys[:c], wdgen.values(c, 17))
+    assert r.ins.new_keys == c and r.ins.failures == 0
+    assert not np.any(r.table == np.uint64(0xFFFFFFFFFFFFFFFF))
+    r.insert(keys[c:], wdgen.values(1, 18))
+    assert r.ins.failures == 1
+
+
 def test_replay_layout_independent_of_group_size_p89():
     # "The inner probing loop (Line 6) ensures a consistent probing scheme in case
     # that the size of g is varied": the sequential layout must not depend on |g|.
@@ -295,7 +344,7 @@ def test_replay_results_equal_map(dup):
     # the replay of Fig. 3 reaches the same map as the plain dictionary (sequential
     # upserts, last value wins), for hits, misses and updates
     n = 20000
-    c = (int(n / 0.95) + 3) // 4 * 4
+    c = oracle.physical_capacity(int(n / 0.95))
     if dup:
         keys = wdgen.uniform_keys(n, 3) % np.uint32(9000)  # many repeats
     else:

@@ -22,11 +22,10 @@ def main(n=1 << 22):
     keys, vals = wdgen.unique_keys(n, 1), wdgen.values(n, 2)
     absent = wdgen.unique_keys(n // 4, 1, start=n)
     out = {"_source": "tools/probe_cost.py: oracle.Replay (sequential Fig. 3, readings C1/C2, "
-                      "sector-aligned 32-slot regions), n = %d unique keys, p_max = 1024" % n,
+                      "sector-aligned 32-slot regions, prime region count), n = %d unique keys, p_max = 1024" % n,
            "rows": []}
     for alpha in (0.8, 0.9, 0.95, 0.99):
-        c = int(math.ceil(n / alpha))
-        c = (c + 3) // 4 * 4
+        c = oracle.physical_capacity(int(math.ceil(n / alpha)))
         for G in (1, 2, 4, 8, 16, 32):
             r = oracle.Replay(c, G)
             r.insert(keys, vals)
