@@ -117,14 +117,20 @@ def peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def cpu_baseline_sample(log2n: int = 24):
+def cpu_baseline_sample(log2n: int = 26):
     """The oracle as it stands (single-threaded C dictionary), on a bounded sample of the
-    same workload: 2^log2n unique inserts + 2^log2n hit queries."""
+    same workload: 2^log2n unique inserts + 2^log2n hit queries (inputs from the same
+    counter-based generator, produced on the device and copied to the host)."""
     import numpy as np
     import oracle
-    import wdgen
     n = 1 << log2n
-    keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
+    try:
+        import wdgen.gpu as gg
+        keys = gg.unique_keys(n, KEY_SEED).cpu().numpy().view(np.uint32)
+        vals = gg.values(n, VAL_SEED).cpu().numpy().view(np.uint32)
+    except Exception:
+        import wdgen
+        keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
     m = oracle.Map(n)
     t0 = time.perf_counter()
     m.insert(keys, vals)

@@ -122,7 +122,8 @@ wd_status_t wd_sync(wd_table_t* t);
 /* ------------------------------------------------------------------ options -------- */
 typedef enum {
     WD_OPT_GROUP_SIZE = 0,   /* |g|; the probe sequence does not depend on it */
-    WD_OPT_P_MAX = 1,        /* outer probing bound p_max (Fig. 3 Line 4), default 1024 (C4) */
+    WD_OPT_P_MAX = 1,        /* outer probing bound p_max (Fig. 3 Line 4); 0 (default) = the
+                                number of regions nb, i.e. fail only when the table is full (C4') */
     WD_OPT_BATCH = 2,        /* items per shard per pipeline batch (2^24) */
     WD_OPT_SERIAL = 3,       /* 1: one probing group, one key at a time (deterministic
                                 layout, test hook for the Fig. 3 replay) */
@@ -149,8 +150,8 @@ uint64_t    wd_shard_capacity(wd_table_t* t, int shard);
  * word = key | (uint64_t)value << 32, empty = all ones.  Synchronizes. */
 wd_status_t wd_dump(wd_table_t* t, int shard, uint64_t* host_out);
 /* per-shard device counters: [0] new keys, [1] failed inserts, [2] reserved keys,
- * [3] exchange errors.  Synchronizes. */
-wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[4]);
+ * [3] exchange errors, [4] key of the most recent failed insert.  Synchronizes. */
+wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[5]);
 
 #ifdef __cplusplus
 }

@@ -223,10 +223,10 @@ class Table:
         return out
 
     def counters(self, shard: int = 0) -> dict:
-        out = np.zeros(4, np.uint64)
+        out = np.zeros(5, np.uint64)
         _check(_lib.wd_counters(self._h, shard, out.ctypes.data))
         return {"new": int(out[0]), "failed": int(out[1]), "reserved": int(out[2]),
-                "exchange_errors": int(out[3])}
+                "exchange_errors": int(out[3]), "last_failed_key": int(out[4])}
 
     @property
     def launches(self) -> int:

@@ -122,7 +122,7 @@ struct wd_table {
   int m = 1;          // number of shards (= GPUs, or virtual shards in loopback)
   int rank = 0;       // rank mode: this process's shard id
   int G = 4;
-  int pmax = 1024;
+  int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit
   int kif = 0;        // keys in flight per group (0 = default)
   uint64_t batch = 1ull << 24;
   int serial = 0;
@@ -182,7 +182,10 @@ template <int G, int K, bool INSERT, class In, class Out>
 wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
   auto kern = wd::probe_kernel<G, K, INSERT, In, Out>;
-  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), static_cast<uint32_t>(t->pmax)};
+  // C4': default p_max = nb — eq. 3 then visits every region, so an insert fails only when
+  // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
+  const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
+  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax};
   int grid = 1, block = 32;
   if (!t->serial) {
     block = wd::kBlock;
@@ -200,7 +203,7 @@ template <int G, bool INSERT, class In, class Out>
 wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
   int k = t->kif;
-  if (k == 0) k = 4;
+  if (k == 0) k = G <= 4 ? 8 : 4;   // measured on B200 (tools/gpu_run3.sh sweep)
   if (k == 4) return launch_probe_k<G, 4, INSERT>(t, s, in, out, n_hint, st);
   return launch_probe_k<G, 8, INSERT>(t, s, in, out, n_hint, st);
 }
@@ -821,7 +824,7 @@ uint64_t shard_cap(uint64_t capacity, int m) {
 }
 
 wd_status_t sticky_status(wd_table* t) {
-  unsigned long long agg[wd::CNT_N] = {0, 0, 0, 0};
+  unsigned long long agg[wd::CNT_N] = {0, 0, 0, 0, 0};
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
     unsigned long long c[wd::CNT_N];
@@ -1055,7 +1058,7 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       t->G = int(v);
       return WD_OK;
     case WD_OPT_P_MAX:
-      if (v < 1 || v > (1 << 20)) return fail(WD_ERR_INVALID_ARG, "p_max %lld", (long long)v);
+      if (v < 0 || v > (1 << 26)) return fail(WD_ERR_INVALID_ARG, "p_max %lld", (long long)v);
       t->pmax = int(v);
       return WD_OK;
     case WD_OPT_BATCH:
@@ -1083,7 +1086,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_P_MAX: return t->pmax;
     case WD_OPT_BATCH: return int64_t(t->batch);
     case WD_OPT_SERIAL: return t->serial;
-    case WD_OPT_KEYS_IN_FLIGHT: return t->kif ? t->kif : 4;
+    case WD_OPT_KEYS_IN_FLIGHT: return t->kif ? t->kif : (t->G <= 4 ? 8 : 4);
     case WD_OPT_PART_SEED: return t->pseed;
     case WD_OPT_PART_MODE: return t->pmode;
     case WD_OPT_N_SHARDS: return t->m;
@@ -1129,13 +1132,13 @@ wd_status_t wd_dump(wd_table_t* t, int shard, uint64_t* host_out) {
   return WD_OK;
 }
 
-wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[4]) {
+wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[5]) {
   if (!t || shard < 0 || shard >= int(t->local.size()) || !out)
     return fail(WD_ERR_INVALID_ARG, "wd_counters arguments");
   Shard& s = t->local[shard];
   DeviceGuard g(s.device);
   CK(cudaDeviceSynchronize());
-  CK(cudaMemcpy(out, s.counters, 4 * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(out, s.counters, wd::CNT_N * 8, cudaMemcpyDeviceToHost));
   return WD_OK;
 }
 

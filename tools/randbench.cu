@@ -1,0 +1,98 @@
+// randbench.cu — measurement tool (not product): the random-access ceiling of a B200 for
+// the hash table's access pattern.  Every "probe" reads one random window of WB bytes
+// aligned to AB bytes inside a large buffer, fetched by WB/8 lanes x 8 B (the coalesced
+// group pattern, |g| = WB/8).  Each lane keeps D independent windows in flight.  Variants:
+//   read : window read only (a query)
+//   cas  : window read, then a 64-bit CAS on the window's first slot that FAILS (no write)
+//   casw : ... a CAS that SUCCEEDS (dirty sector, written back later: an insert)
+// Reports windows/s and useful GB/s for 2.26 GB (config 2 table) and 36 GB buffers.
+// Build: nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o tools/randbench tools/randbench.cu
+#include <cstdio>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+__device__ __forceinline__ uint32_t hash32(uint32_t x) {
+  x ^= x >> 16; x *= 0x7feb352du; x ^= x >> 15; x *= 0x846ca68bu; x ^= x >> 16;
+  return x;
+}
+__device__ __forceinline__ unsigned long long ldr(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+
+template <int D, int MODE, int WB, int AB>
+__global__ void __launch_bounds__(256) gather(unsigned long long* buf, uint64_t nwin, int iters,
+                                              uint32_t salt, unsigned long long* sink) {
+  constexpr int L = WB / 8;  // lanes per window
+  const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t g = tid / L, r = tid % L;
+  unsigned long long acc = 0;
+  for (int it = 0; it < iters; ++it) {
+    unsigned long long v[D];
+    const unsigned long long* p[D];
+#pragma unroll
+    for (int d = 0; d < D; ++d) {
+      const uint32_t h = hash32(g * 2654435761u + (it * D + d) * 40503u + salt);
+      const uint64_t w = (uint64_t(h) * nwin) >> 32;         // window start = w * AB bytes
+      p[d] = buf + w * (AB / 8) + r;
+      v[d] = ldr(p[d]);
+    }
+#pragma unroll
+    for (int d = 0; d < D; ++d) {
+      acc += v[d];
+      if (MODE != 0 && r == 0) {
+        if (MODE == 1) acc += atomicCAS((unsigned long long*)p[d], 0x1234567812345678ull, 1ull);
+        else acc += atomicCAS((unsigned long long*)p[d], v[d], v[d] ^ 1ull);
+      }
+    }
+  }
+  if (acc == 42) sink[0] = acc;
+}
+
+template <int D, int MODE, int WB, int AB>
+void run(const char* name, unsigned long long* buf, uint64_t bytes, int grid, int iters,
+         unsigned long long* sink) {
+  const uint64_t nwin = (bytes - 256) / AB;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a); cudaEventCreate(&b);
+  gather<D, MODE, WB, AB><<<grid, 256>>>(buf, nwin, 2, 1, sink);
+  cudaEventRecord(a);
+  gather<D, MODE, WB, AB><<<grid, 256>>>(buf, nwin, iters, 7, sink);
+  cudaEventRecord(b);
+  cudaEventSynchronize(b);
+  float ms; cudaEventElapsedTime(&ms, a, b);
+  const double windows = double(grid) * 256 / (WB / 8) * D * iters;
+  printf("%.2fGB %-5s W=%3dB align=%3dB D=%d : %6.1f Gwin/s  %6.0f GB/s useful\n", bytes / 1e9, name,
+         WB, AB, D, windows / (ms * 1e-3) / 1e9, windows * WB / (ms * 1e-3) / 1e9);
+}
+
+int main() {
+  int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+  unsigned long long* sink; cudaMalloc(&sink, 8);
+  cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, 32);
+  for (double gb : {2.26, 36.0}) {
+    const uint64_t bytes = uint64_t(gb * 1e9) / 256 * 256;
+    unsigned long long* buf;
+    if (cudaMalloc(&buf, bytes) != cudaSuccess) { printf("alloc %.1f GB failed\n", gb); continue; }
+    cudaMemset(buf, 0xff, bytes);
+    const int grid = sms * 8;
+    const int it = 32;
+    run<8, 0, 8, 32>("read", buf, bytes, grid, it, sink);
+    run<8, 0, 32, 32>("read", buf, bytes, grid, it, sink);
+    run<8, 0, 32, 64>("read", buf, bytes, grid, it, sink);
+    run<8, 0, 64, 32>("read", buf, bytes, grid, it, sink);
+    run<8, 0, 64, 64>("read", buf, bytes, grid, it, sink);
+    run<8, 0, 128, 32>("read", buf, bytes, grid, it, sink);
+    run<8, 0, 128, 128>("read", buf, bytes, grid, it, sink);
+    run<8, 0, 256, 32>("read", buf, bytes, grid, it, sink);
+    run<8, 0, 256, 256>("read", buf, bytes, grid, it, sink);
+    run<8, 1, 32, 32>("cas", buf, bytes, grid, it, sink);
+    run<8, 2, 32, 32>("casw", buf, bytes, grid, it, sink);
+    run<8, 1, 64, 64>("cas", buf, bytes, grid, it, sink);
+    run<8, 2, 64, 64>("casw", buf, bytes, grid, it, sink);
+    cudaFree(buf);
+  }
+  printf("err: %s\n", cudaGetErrorString(cudaGetLastError()));
+  return 0;
+}
