@@ -341,7 +341,7 @@ def main():
     # ---- CPU baseline (rank 0, N = 1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
-        cpu = cpu_baseline_sample(24)
+        cpu = cpu_baseline_sample()
 
     sweep_lines = []
     if args.sweep and world == 1:
