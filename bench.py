@@ -53,6 +53,10 @@ def parse():
     ap.add_argument("--kif", type=int, default=0, help="keys in flight per group (0=default)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--dist-backend", default="nccl",
+                    help="torch.distributed backend for the control plane (gloo: tests)")
+    ap.add_argument("--same-device", action="store_true",
+                    help="all ranks on cuda:0 (dry run of the N>1 path on a 1-GPU box)")
     ap.add_argument("--sweep", action="store_true",
                     help="extra lines: config-2 alpha x |g| sweep (not the headline)")
     return ap.parse_args()
@@ -198,19 +202,19 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     assert world == args.gpus or world == 1, "launch N>1 with torchrun --nproc-per-node N"
-    torch.cuda.set_device(local_rank)
+    dev = 0 if args.same_device else local_rank
+    torch.cuda.set_device(dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group(args.dist_backend)
 
     n = 1 << args.n_log2
     G = args.group_size
     cap_local = int(math.ceil(n / args.alpha))
     if world > 1:
-        uid = wd.Table.unique_id() if rank == 0 else None
-        obj = [uid]
-        dist.broadcast_object_list(obj, src=0)
-        table = wd.Table(cap_local * world, group_size=G, rank=rank, world=world,
-                         unique_id=obj[0])
+        table = wd.Table(cap_local * world, group_size=G, rank=rank, world=world)
     else:
         table = wd.Table(cap_local, 1, G)
     if args.kif:
@@ -230,12 +234,7 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
-    def max_over_ranks(x: float) -> float:
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+    from paper_conf_ipps_junger0s18_b200.dist import max_over_ranks
 
     ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
 
@@ -265,7 +264,7 @@ def main():
     launches0 = table.launches
     marks = [[ev(), ev(), ev()] for _ in range(args.steps)]
     e0, e1 = ev(), ev()
-    with ClockSampler(local_rank) as clk:
+    with ClockSampler(dev) as clk:
         barrier()
         e0.record(stream)
         for k in range(args.steps):

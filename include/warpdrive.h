@@ -48,7 +48,7 @@ typedef enum {
     WD_ERR_INVALID_ARG = 1,
     WD_ERR_OUT_OF_MEMORY = 2,
     WD_ERR_CUDA = 3,
-    WD_ERR_NCCL = 4,
+    WD_ERR_NCCL = 4,           /* reserved (the exchange does not use NCCL) */
     WD_ERR_TABLE_FULL = 5,     /* >=1 insert exhausted p_max regions (Fig. 3 Line 26);
                                   that pair was dropped */
     WD_ERR_RESERVED_KEY = 6,   /* >=1 input key == WD_EMPTY_KEY; those pairs were skipped
@@ -79,13 +79,25 @@ wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size);
  * that happen to be local.  Semantics identical to wd_create(capacity, m, g). */
 wd_table_t* wd_create_loopback(uint64_t capacity, int n_shards, int group_size);
 
-/* One process per GPU (torchrun).  Rank 0 calls wd_get_unique_id and the 128 bytes are
- * broadcast by the caller (torch.distributed); every rank then calls wd_create_rank on
- * its current device.  Collective: all ranks must call every wd_insert / wd_retrieve /
- * wd_clear / wd_size / wd_destroy in the same order (each with its own local n >= 0). */
-wd_status_t wd_get_unique_id(uint8_t unique_id[128]);
-wd_table_t* wd_create_rank(uint64_t capacity, int rank, int world, const uint8_t unique_id[128],
-                           int group_size);
+/* One process per GPU (torchrun).  Collective: every rank calls every wd_insert /
+ * wd_retrieve / wd_clear / wd_size / wd_destroy in the same order (each with its own
+ * local n >= 0).  Bootstrap, on each rank's current device:
+ *   t = wd_create_rank(capacity, rank, world, g);      capacity = total slots, all ranks
+ *   wd_rank_handle(t, blob);                           IPC handle of the exchange arena
+ *   (caller all-gathers the world blobs in rank order, e.g. torch.distributed)
+ *   wd_rank_connect(t, blobs, allreduce, ctx);         maps every peer's arena (NVLink)
+ * `allreduce` is a HOST collective over the same ranks (sum or max of one uint64, in
+ * place, returns 0 on success); it is called synchronously, in the same order on every
+ * rank, for control only (batch-count agreement, wd_size, barriers) — the data path is
+ * peer-memory stores/loads inside the kernels.  WD_OPT_BATCH is fixed once connected. */
+#define WD_RANK_HANDLE_BYTES 128
+#define WD_REDUCE_SUM 0
+#define WD_REDUCE_MAX 1
+typedef int (*wd_allreduce_fn)(uint64_t* value, int op, void* ctx);
+wd_table_t* wd_create_rank(uint64_t capacity, int rank, int world, int group_size);
+wd_status_t wd_rank_handle(wd_table_t* t, uint8_t out[WD_RANK_HANDLE_BYTES]);
+wd_status_t wd_rank_connect(wd_table_t* t, const uint8_t* handles, wd_allreduce_fn allreduce,
+                            void* ctx);
 
 /* NULL-safe.  Synchronizes, then frees table, buffers, peer mappings and communicators. */
 void wd_destroy(wd_table_t* t);

@@ -30,8 +30,12 @@ WD_NOT_FOUND = 0xFFFFFFFF
 WD_OPT_GROUP_SIZE, WD_OPT_P_MAX, WD_OPT_BATCH, WD_OPT_SERIAL = 0, 1, 2, 3
 WD_OPT_KEYS_IN_FLIGHT, WD_OPT_PART_SEED, WD_OPT_PART_MODE = 4, 5, 6
 WD_OPT_N_SHARDS, WD_OPT_RANK, WD_OPT_LOCAL_SHARDS, WD_OPT_LAUNCHES = 100, 101, 102, 103
+WD_RANK_HANDLE_BYTES = 128
+# int (*)(uint64_t* value, int op, void* ctx)
+ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.POINTER(C.c_uint64), C.c_int, C.c_void_p)
 
-EXPORTS = ["wd_create", "wd_create_loopback", "wd_get_unique_id", "wd_create_rank",
+EXPORTS = ["wd_create", "wd_create_loopback", "wd_create_rank", "wd_rank_handle",
+           "wd_rank_connect",
            "wd_destroy", "wd_clear", "wd_insert", "wd_retrieve", "wd_size", "wd_capacity",
            "wd_sync", "wd_set_option", "wd_get_option", "wd_last_error", "wd_error_string",
            "wd_last_error_message", "wd_shard_capacity", "wd_dump", "wd_counters"]
@@ -59,8 +63,9 @@ def _load():
     sig = {
         "wd_create": ([u64, i32, i32], p),
         "wd_create_loopback": ([u64, i32, i32], p),
-        "wd_get_unique_id": ([p], i32),
-        "wd_create_rank": ([u64, i32, i32, p, i32], p),
+        "wd_create_rank": ([u64, i32, i32, i32], p),
+        "wd_rank_handle": ([p, p], i32),
+        "wd_rank_connect": ([p, p, p, p], i32),
         "wd_destroy": ([p], None),
         "wd_clear": ([p, p], i32),
         "wd_insert": ([p, p, p, u64, p], i32),
@@ -127,25 +132,41 @@ class Table:
 
     def __init__(self, capacity: int, n_gpus: int = 1, group_size: int = 4, *,
                  loopback_shards: int | None = None, rank: int | None = None,
-                 world: int | None = None, unique_id: bytes | None = None):
+                 world: int | None = None, process_group=None, batch: int | None = None):
+        """rank/world: one process per GPU (torchrun); the exchange handles are all-gathered
+        and the host collective is run over `process_group` (torch.distributed)."""
+        self._cb = None
         if loopback_shards is not None:
             h = _lib.wd_create_loopback(int(capacity), int(loopback_shards), int(group_size))
         elif rank is not None:
-            assert world is not None and unique_id is not None and len(unique_id) == 128
-            buf = (C.c_uint8 * 128).from_buffer_copy(unique_id)
-            h = _lib.wd_create_rank(int(capacity), int(rank), int(world), C.addressof(buf),
-                                    int(group_size))
+            assert world is not None
+            h = _lib.wd_create_rank(int(capacity), int(rank), int(world), int(group_size))
         else:
             h = _lib.wd_create(int(capacity), int(n_gpus), int(group_size))
         if not h:
             raise WarpDriveError(_lib.wd_last_error(), _lib.wd_last_error_message().decode())
         self._h = h
+        if batch is not None:
+            self.set_option(WD_OPT_BATCH, batch)
+        if rank is not None:
+            self._connect(process_group)
 
-    @staticmethod
-    def unique_id() -> bytes:
-        buf = (C.c_uint8 * 128)()
-        _check(_lib.wd_get_unique_id(C.addressof(buf)))
-        return bytes(buf)
+    def _connect(self, group):
+        from . import dist as wdist
+        blob = (C.c_uint8 * WD_RANK_HANDLE_BYTES)()
+        _check(_lib.wd_rank_handle(self._h, C.addressof(blob)))
+        blobs = wdist.allgather_bytes(bytes(blob), group)
+        allb = (C.c_uint8 * (WD_RANK_HANDLE_BYTES * len(blobs))).from_buffer_copy(b"".join(blobs))
+
+        def _allreduce(vptr, op, ctx):
+            try:
+                vptr[0] = wdist.allreduce_u64(int(vptr[0]), int(op), group)
+                return 0
+            except Exception:  # pragma: no cover - reported as WD_ERR_EXCHANGE
+                return 1
+
+        self._cb = ALLREDUCE_FN(_allreduce)   # keep alive as long as the table
+        _check(_lib.wd_rank_connect(self._h, C.addressof(allb), self._cb, None))
 
     # -- lifetime
     def close(self):

@@ -3,7 +3,8 @@
   paper_conf_ipps_junger0s18_b200/libwarpdrive.so   the product (C-ABI, include/warpdrive.h)
   wdgen/libwdgen.so                                  device-side input generator (bench/tests)
 
-NCCL is the copy shipped in the venv (nvidia/nccl, 2.28), the one torch loads.
+The multi-GPU exchange is peer-memory stores/loads inside the kernels (CUDA IPC for one
+process per GPU), so the library links only the CUDA runtime.
 """
 from __future__ import annotations
 
@@ -20,12 +21,6 @@ COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
 
 LIB = os.path.join(PKG, "libwarpdrive.so")
 GENLIB = os.path.join(ROOT, "wdgen", "libwdgen.so")
-
-
-def nccl_paths():
-    import nvidia.nccl as n  # noqa: the venv's NCCL (torch's)
-    base = list(n.__path__)[0]
-    return os.path.join(base, "include"), os.path.join(base, "lib")
 
 
 def _stale(out, srcs):
@@ -45,11 +40,9 @@ def build(force: bool = False, verbose: bool = False, extra: list[str] | None = 
     srcs = [os.path.join(PKG, "csrc", "warpdrive.cu"), os.path.join(PKG, "csrc", "wd_device.cuh"),
             os.path.join(ROOT, "include", "warpdrive.h")]
     if force or _stale(LIB, srcs):
-        inc, lib = nccl_paths()
         tmp = LIB + f".tmp{os.getpid()}"
         _run([NVCC, *ARCH, *COMMON, *(extra or []), "-I", os.path.join(ROOT, "include"),
-              "-I", inc, "-o", tmp, srcs[0], "-L", lib, "-l:libnccl.so.2",
-              "-Xlinker", f"-rpath,{lib}"], verbose)
+              "-o", tmp, srcs[0]], verbose)
         os.replace(tmp, LIB)
     gsrc = [os.path.join(ROOT, "wdgen", "wdgen.cu")]
     if force or _stale(GENLIB, gsrc):

@@ -15,7 +15,6 @@
 //                     result regions are double-buffered by epoch parity.
 // =====================================================================================
 #include <cuda_runtime.h>
-#include <nccl.h>
 
 #include <algorithm>
 #include <cstdarg>
@@ -48,13 +47,6 @@ wd_status_t fail(wd_status_t s, const char* fmt, ...) {
     if (e_ != cudaSuccess)                                                               \
       return fail(e_ == cudaErrorMemoryAllocation ? WD_ERR_OUT_OF_MEMORY : WD_ERR_CUDA,  \
                   "%s: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, __LINE__);     \
-  } while (0)
-#define NK(x)                                                                            \
-  do {                                                                                   \
-    ncclResult_t r_ = (x);                                                               \
-    if (r_ != ncclSuccess)                                                               \
-      return fail(WD_ERR_NCCL, "%s: %s (%s:%d)", #x, ncclGetErrorString(r_), __FILE__,   \
-                  __LINE__);                                                             \
   } while (0)
 #define TRY(x)                          \
   do {                                  \
@@ -136,8 +128,10 @@ struct wd_table {
   std::vector<Shard> local;
   std::vector<PeerView> peers;  // size m
   std::vector<void*> opened;    // IPC-mapped peer arenas (rank mode)
-  ncclComm_t comm = nullptr;
-  unsigned long long* d_scratch = nullptr;  // rank mode: allreduce scratch
+  // rank mode: host collective supplied by the caller (torch.distributed), connected peers
+  wd_allreduce_fn allreduce = nullptr;
+  void* allreduce_ctx = nullptr;
+  bool connected = false;
   cudaStream_t loop_stream = nullptr;       // loopback: one stream for all shards
 };
 
@@ -393,6 +387,8 @@ wd_status_t rank_allgather_views(wd_table* t, uint64_t B);
 wd_status_t ensure_exchange(wd_table* t) {
   if (t->m == 1) return WD_OK;
   if (t->xbatch == t->batch) return WD_OK;
+  if (t->mode == MODE_RANK && t->connected)
+    return fail(WD_ERR_INVALID_ARG, "rank mode: batch size fixed after wd_rank_connect");
   const uint64_t B = t->batch;
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
@@ -404,7 +400,8 @@ wd_status_t ensure_exchange(wd_table* t) {
   for (auto& s : t->local) TRY(exchange_init_shard(t, s, B));
   t->peers.assign(t->m, PeerView{});
   if (t->mode == MODE_RANK) {
-    TRY(rank_allgather_views(t, B));
+    if (t->connected) return fail(WD_ERR_INVALID_ARG, "rank mode: batch size fixed after wd_rank_connect");
+    t->peers[t->rank] = t->local[0].self;   // peers mapped by wd_rank_connect
   } else {
     for (auto& s : t->local) t->peers[s.id] = s.self;
   }
@@ -414,33 +411,21 @@ wd_status_t ensure_exchange(wd_table* t) {
   return WD_OK;
 }
 
-wd_status_t rank_allgather_views(wd_table* t, uint64_t B) {
-  Shard& s = t->local[0];
-  DeviceGuard g(s.device);
-  cudaIpcMemHandle_t h;
-  CK(cudaIpcGetMemHandle(&h, s.arena));
-  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "ipc handle size");
-  char* d_buf = nullptr;
-  CK(cudaMalloc(&d_buf, size_t(64) * t->m));
-  CK(cudaMemcpy(d_buf + 64 * t->rank, &h, 64, cudaMemcpyHostToDevice));
-  NK(ncclAllGather(d_buf + 64 * t->rank, d_buf, 64, ncclChar, t->comm, s.s_main));
-  std::vector<cudaIpcMemHandle_t> all(t->m);
-  CK(cudaMemcpyAsync(all.data(), d_buf, size_t(64) * t->m, cudaMemcpyDeviceToHost, s.s_main));
-  CK(cudaStreamSynchronize(s.s_main));
-  cudaFree(d_buf);
-  for (int d = 0; d < t->m; ++d) {
-    if (d == t->rank) {
-      t->peers[d] = s.self;
-      continue;
-    }
-    void* base = nullptr;
-    CK(cudaIpcOpenMemHandle(&base, all[d], cudaIpcMemLazyEnablePeerAccess));
-    t->opened.push_back(base);
-    t->peers[d] = arena_view(base, t->m, B);
-  }
-  // everyone mapped everyone before first use
-  NK(ncclAllReduce(t->d_scratch, t->d_scratch, 1, ncclUint64, ncclSum, t->comm, s.s_main));
-  CK(cudaStreamSynchronize(s.s_main));
+// rank-mode handle blob: IPC handle of the exchange arena + its geometry
+struct RankHandle {
+  char ipc[64];
+  uint64_t magic, batch, arena_bytes;
+  uint32_t world, rank;
+  char pad[WD_RANK_HANDLE_BYTES - 64 - 3 * 8 - 2 * 4];
+};
+static_assert(sizeof(RankHandle) == WD_RANK_HANDLE_BYTES, "rank handle size");
+constexpr uint64_t kHandleMagic = 0x5744524B48444C31ull;  // "WDRKHDL1"
+
+wd_status_t host_allreduce(wd_table* t, uint64_t* v, int op) {
+  if (t->mode != MODE_RANK) return WD_OK;
+  if (!t->allreduce) return fail(WD_ERR_INVALID_ARG, "rank mode: not connected (wd_rank_connect)");
+  if (t->allreduce(v, op, t->allreduce_ctx) != 0)
+    return fail(WD_ERR_EXCHANGE, "rank mode: host allreduce callback failed");
   return WD_OK;
 }
 
@@ -609,17 +594,8 @@ wd_status_t launch_signal(wd_table* t, Shard& s, int flag, unsigned long long ep
 }
 
 wd_status_t agree_batches(wd_table* t, uint64_t local_nbt, uint64_t* global_nbt) {
-  if (t->mode != MODE_RANK) {
-    *global_nbt = local_nbt;
-    return WD_OK;
-  }
-  Shard& s = t->local[0];
-  DeviceGuard g(s.device);
-  unsigned long long v = local_nbt;
-  CK(cudaMemcpyAsync(t->d_scratch, &v, 8, cudaMemcpyHostToDevice, s.s_main));
-  NK(ncclAllReduce(t->d_scratch, t->d_scratch, 1, ncclUint64, ncclMax, t->comm, s.s_main));
-  CK(cudaMemcpyAsync(&v, t->d_scratch, 8, cudaMemcpyDeviceToHost, s.s_main));
-  CK(cudaStreamSynchronize(s.s_main));
+  uint64_t v = local_nbt;
+  TRY(host_allreduce(t, &v, WD_REDUCE_MAX));   // every rank runs the same batch sequence
   *global_nbt = v;
   return WD_OK;
 }
@@ -910,17 +886,8 @@ wd_table_t* wd_create_loopback(uint64_t capacity, int n_shards, int group_size) 
   return t;
 }
 
-wd_status_t wd_get_unique_id(uint8_t unique_id[128]) {
-  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
-  ncclUniqueId id;
-  NK(ncclGetUniqueId(&id));
-  memcpy(unique_id, &id, 128);
-  return WD_OK;
-}
-
-wd_table_t* wd_create_rank(uint64_t capacity, int rank, int world, const uint8_t unique_id[128],
-                           int group_size) {
-  if (world < 1 || rank < 0 || rank >= world || !unique_id) {
+wd_table_t* wd_create_rank(uint64_t capacity, int rank, int world, int group_size) {
+  if (world < 1 || rank < 0 || rank >= world) {
     fail(WD_ERR_INVALID_ARG, "rank %d / world %d", rank, world);
     return nullptr;
   }
@@ -939,23 +906,62 @@ wd_table_t* wd_create_rank(uint64_t capacity, int rank, int world, const uint8_t
     wd_destroy(t);
     return nullptr;
   }
-  if (world > 1) {
-    ncclUniqueId id;
-    memcpy(&id, unique_id, 128);
-    ncclResult_t r = ncclCommInitRank(&t->comm, world, id, rank);
-    if (r != ncclSuccess) {
-      fail(WD_ERR_NCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
-      wd_destroy(t);
-      return nullptr;
-    }
-    if (cudaMalloc(&t->d_scratch, 64) != cudaSuccess || ensure_exchange(t) != WD_OK) {
-      if (g_last == WD_OK) fail(WD_ERR_OUT_OF_MEMORY, "scratch allocation");
-      wd_destroy(t);
-      return nullptr;
-    }
-  }
   g_last = WD_OK;
   return t;
+}
+
+wd_status_t wd_rank_handle(wd_table_t* t, uint8_t out[WD_RANK_HANDLE_BYTES]) {
+  if (!t || !out) return fail(WD_ERR_INVALID_ARG, "wd_rank_handle arguments");
+  RankHandle h;
+  memset(&h, 0, sizeof h);
+  h.magic = kHandleMagic;
+  h.world = uint32_t(t->m);
+  h.rank = uint32_t(t->rank);
+  if (t->mode == MODE_RANK) {
+    TRY(ensure_exchange(t));                  // arena for the current batch size
+    Shard& s = t->local[0];
+    DeviceGuard g(s.device);
+    cudaIpcMemHandle_t ipc;
+    CK(cudaIpcGetMemHandle(&ipc, s.arena));
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "ipc handle size");
+    memcpy(h.ipc, &ipc, 64);
+    h.batch = t->xbatch;
+    h.arena_bytes = s.arena_bytes;
+  }
+  memcpy(out, &h, sizeof h);
+  return WD_OK;
+}
+
+wd_status_t wd_rank_connect(wd_table_t* t, const uint8_t* handles, wd_allreduce_fn fn, void* ctx) {
+  if (!t || !handles || !fn) return fail(WD_ERR_INVALID_ARG, "wd_rank_connect arguments");
+  t->allreduce = fn;
+  t->allreduce_ctx = ctx;
+  if (t->mode != MODE_RANK) { t->connected = true; return WD_OK; }
+  if (t->connected) return fail(WD_ERR_INVALID_ARG, "already connected");
+  TRY(ensure_exchange(t));
+  Shard& s = t->local[0];
+  DeviceGuard g(s.device);
+  for (int d = 0; d < t->m; ++d) {
+    RankHandle h;
+    memcpy(&h, handles + size_t(d) * WD_RANK_HANDLE_BYTES, sizeof h);
+    if (h.magic != kHandleMagic || int(h.world) != t->m || int(h.rank) != d)
+      return fail(WD_ERR_INVALID_ARG, "handle %d: bad magic/world/rank order", d);
+    if (h.batch != t->xbatch || h.arena_bytes != s.arena_bytes)
+      return fail(WD_ERR_INVALID_ARG, "handle %d: batch size differs between ranks", d);
+    if (d == t->rank) continue;
+    cudaIpcMemHandle_t ipc;
+    memcpy(&ipc, h.ipc, 64);
+    void* base = nullptr;
+    CK(cudaIpcOpenMemHandle(&base, ipc, cudaIpcMemLazyEnablePeerAccess));
+    t->opened.push_back(base);
+    t->peers[d] = arena_view(base, t->m, t->xbatch);
+  }
+  t->connected = true;
+  uint64_t one = 1;                            // every rank mapped every peer before use
+  TRY(host_allreduce(t, &one, WD_REDUCE_SUM));
+  if (one != uint64_t(t->m)) return fail(WD_ERR_EXCHANGE, "connect barrier: %llu of %d ranks",
+                                         (unsigned long long)one, t->m);
+  return WD_OK;
 }
 
 void wd_destroy(wd_table_t* t) {
@@ -964,15 +970,12 @@ void wd_destroy(wd_table_t* t) {
     DeviceGuard g(s.device);
     cudaDeviceSynchronize();
   }
-  if (t->comm) {  // collective: no rank unmaps before every rank is done
-    ncclAllReduce(t->d_scratch, t->d_scratch, 1, ncclUint64, ncclSum, t->comm,
-                  t->local[0].s_main);
-    cudaStreamSynchronize(t->local[0].s_main);
+  if (t->mode == MODE_RANK && t->connected) {  // no rank unmaps before every rank is done
+    uint64_t one = 1;
+    host_allreduce(t, &one, WD_REDUCE_SUM);
   }
   for (void* p : t->opened) cudaIpcCloseMemHandle(p);
   for (auto& s : t->local) shard_free(s);
-  if (t->comm) ncclCommDestroy(t->comm);
-  if (t->d_scratch) cudaFree(t->d_scratch);
   if (t->loop_stream) cudaStreamDestroy(t->loop_stream);
   delete t;
 }
@@ -1030,16 +1033,9 @@ uint64_t wd_size(wd_table_t* t) {
     total += c;
   }
   if (t->mode == MODE_RANK) {
-    Shard& s = t->local[0];
-    DeviceGuard g(s.device);
-    if (cudaMemcpy(t->d_scratch, &total, 8, cudaMemcpyHostToDevice) != cudaSuccess ||
-        ncclAllReduce(t->d_scratch, t->d_scratch, 1, ncclUint64, ncclSum, t->comm, s.s_main) !=
-            ncclSuccess ||
-        cudaStreamSynchronize(s.s_main) != cudaSuccess ||
-        cudaMemcpy(&total, t->d_scratch, 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
-      fail(WD_ERR_NCCL, "wd_size allreduce failed");
-      return UINT64_MAX;
-    }
+    uint64_t v = total;
+    if (host_allreduce(t, &v, WD_REDUCE_SUM) != WD_OK) return UINT64_MAX;
+    total = v;
   }
   return total;
 }

@@ -1,0 +1,66 @@
+"""CPU checks of the boundary: the C-ABI library loads and exports every function that
+include/warpdrive.h declares (no compute calls), and the Python binding carries the same
+names.  Also: the oracle and generator libraries build and load."""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "warpdrive.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(wd_[a-z_]+)\s*\(", src)) - {"wd_allreduce_fn"})
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_ipps_junger0s18_b200 import build
+    build.build()
+    return ctypes.CDLL(build.LIB)
+
+
+def test_header_declares_the_north_star_calls():
+    names = _declared()
+    for n in ["wd_create", "wd_insert", "wd_retrieve", "wd_size", "wd_destroy"]:
+        assert n in names
+
+
+def test_library_exports_every_declared_symbol(lib):
+    missing = [n for n in _declared() if not hasattr(lib, n)]
+    assert not missing, missing
+
+
+def test_binding_names_match_header(lib):
+    import paper_conf_ipps_junger0s18_b200 as wd
+    assert sorted(wd.EXPORTS) == _declared()
+    for n in wd.EXPORTS:
+        assert callable(getattr(wd, n))
+
+
+def test_error_strings_without_gpu(lib):
+    import paper_conf_ipps_junger0s18_b200 as wd
+    assert wd.wd_error_string(wd.WD_ERR_TABLE_FULL) == b"WD_ERR_TABLE_FULL"
+    assert wd.wd_error_string(0) == b"WD_OK"
+
+
+def test_sm100a_only_and_no_cpu_fallback(lib):
+    # the product library contains sm_100a SASS only
+    import subprocess
+    from paper_conf_ipps_junger0s18_b200 import build
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", build.LIB],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    assert all("sm_100a" in line for line in out.splitlines() if ".cubin" in line)
+
+
+def test_oracle_and_generator_libraries_load():
+    import oracle
+    assert os.path.exists(oracle.build())
+    from paper_conf_ipps_junger0s18_b200 import build
+    build.build()
+    g = ctypes.CDLL(build.GENLIB)
+    assert hasattr(g, "wdgen_unique_keys")
