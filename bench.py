@@ -51,6 +51,8 @@ def parse():
     ap.add_argument("--alpha", type=float, default=0.95)
     ap.add_argument("--group-size", type=int, default=4)
     ap.add_argument("--kif", type=int, default=0, help="keys in flight per group (0=default)")
+    ap.add_argument("--probe-mode", type=int, default=None,
+                    help="0: cooperative group per window (Fig. 3); 1: lane-window")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--dist-backend", default="nccl",
@@ -219,6 +221,8 @@ def main():
         table = wd.Table(cap_local, 1, G)
     if args.kif:
         table.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, args.kif)
+    if args.probe_mode is not None:
+        table.set_option(wd.WD_OPT_PROBE_MODE, args.probe_mode)
 
     # inputs: rank r inserts generator indices [r n, (r+1) n) -> globally unique keys
     keys = gg.unique_keys(n, KEY_SEED, start=rank * n)

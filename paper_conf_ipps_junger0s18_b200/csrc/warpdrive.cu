@@ -116,6 +116,7 @@ struct wd_table {
   int G = 4;
   int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit
   int kif = 0;        // keys in flight per group (0 = default)
+  int probe_mode = 0; // 0: cooperative groups (Fig. 3), 1: lane-window (|g| <= 8)
   uint64_t batch = 1ull << 24;
   int serial = 0;
   uint32_t pseed = 0x9E3779B9u;
@@ -193,11 +194,55 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
   return WD_OK;
 }
 
+template <int G, int K, bool INSERT, class In, class Out>
+wd_status_t launch_lane_k(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
+                          cudaStream_t st) {
+  auto kern = wd::probe_lane_kernel<G, K, INSERT, In, Out>;
+  const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
+  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax};
+  int grid = 1, block = 32;
+  if (!t->serial) {
+    block = wd::kBlock;
+    const uint64_t keys_per_block = uint64_t(wd::kBlock) * K;
+    const uint64_t need = std::max<uint64_t>(1, (n_hint + keys_per_block - 1) / keys_per_block);
+    grid = static_cast<int>(std::min<uint64_t>(need, uint64_t(t->sm_count) * blocks_per_sm(kern)));
+  }
+  kern<<<grid, block, 0, st>>>(tv, in, out, s.counters, t->serial);
+  CK(cudaGetLastError());
+  t->launches++;
+  return WD_OK;
+}
+
+// lane-window keys in flight per lane: window registers grow with |g| (8|g| bytes each)
+int lane_k(int G, int kif) {
+  if (kif == 1 || kif == 2 || kif == 4 || kif == 8) {
+    if (G >= 8 && kif == 8) return 4;
+    return kif;
+  }
+  if (G >= 8) return 2;
+  if (G == 4) return 4;
+  return 8;
+}
+
 template <int G, bool INSERT, class In, class Out>
 wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
+  if constexpr (G <= 8) {
+    if (t->probe_mode == 1) {
+      const int k = lane_k(G, t->kif);
+      if (k == 1) return launch_lane_k<G, 1, INSERT>(t, s, in, out, n_hint, st);
+      if (k == 2) return launch_lane_k<G, 2, INSERT>(t, s, in, out, n_hint, st);
+      if constexpr (G == 8) {
+        return launch_lane_k<G, 4, INSERT>(t, s, in, out, n_hint, st);
+      } else {
+        if (k == 8) return launch_lane_k<G, 8, INSERT>(t, s, in, out, n_hint, st);
+        return launch_lane_k<G, 4, INSERT>(t, s, in, out, n_hint, st);
+      }
+    }
+  }
   int k = t->kif;
   if (k == 0) k = G <= 4 ? 8 : 4;   // measured on B200 (tools/gpu_run3.sh sweep)
+  if (k == 2) return launch_probe_k<G, 2, INSERT>(t, s, in, out, n_hint, st);
   if (k == 4) return launch_probe_k<G, 4, INSERT>(t, s, in, out, n_hint, st);
   return launch_probe_k<G, 8, INSERT>(t, s, in, out, n_hint, st);
 }
@@ -1063,10 +1108,14 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       return WD_OK;
     case WD_OPT_SERIAL: t->serial = v ? 1 : 0; return WD_OK;
     case WD_OPT_KEYS_IN_FLIGHT:
-      if (v != 0 && v != 4 && v != 8) return fail(WD_ERR_INVALID_ARG, "keys in flight %lld", (long long)v);
+      if (v != 0 && v != 1 && v != 2 && v != 4 && v != 8) return fail(WD_ERR_INVALID_ARG, "keys in flight %lld", (long long)v);
       t->kif = int(v);
       return WD_OK;
     case WD_OPT_PART_SEED: t->pseed = uint32_t(v); return WD_OK;
+    case WD_OPT_PROBE_MODE:
+      if (v != 0 && v != 1) return fail(WD_ERR_INVALID_ARG, "probe mode %lld", (long long)v);
+      t->probe_mode = int(v);
+      return WD_OK;
     case WD_OPT_PART_MODE:
       if (v != 0 && v != 1) return fail(WD_ERR_INVALID_ARG, "partition mode %lld", (long long)v);
       t->pmode = int(v);
@@ -1084,6 +1133,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_SERIAL: return t->serial;
     case WD_OPT_KEYS_IN_FLIGHT: return t->kif ? t->kif : (t->G <= 4 ? 8 : 4);
     case WD_OPT_PART_SEED: return t->pseed;
+    case WD_OPT_PROBE_MODE: return t->probe_mode;
     case WD_OPT_PART_MODE: return t->pmode;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;

@@ -23,12 +23,13 @@ def wd():
 
 
 @pytest.mark.parametrize("m", [2, 3, 4, 8])
-@pytest.mark.parametrize("G", [1, 4, 32])
-def test_loopback_unique_parity(wd, m, G):
+@pytest.mark.parametrize("G,mode", [(1, 0), (4, 0), (32, 0), (4, 1)])
+def test_loopback_unique_parity(wd, m, G, mode):
     n = 200_000 + 17 * m
     keys, vals = wdgen.unique_keys(n, 21), wdgen.values(n, 22)
     q = wdgen.interleaved_queries(n, 21)
     with wd.Table(capacity_for(n, 0.9), group_size=G, loopback_shards=m) as t:
+        t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_BATCH, 9_000)  # many batches per shard: epochs wrap slots
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0, wd._lib.wd_last_error_message()

@@ -27,13 +27,17 @@ def _oracle_answers(keys, vals, queries, dup=False):
     return m, *m.retrieve(queries)
 
 
-@pytest.mark.parametrize("G", GS)
-def test_config1_unique_parity(wd, G):
+MODES = [(G, 0) for G in GS] + [(G, 1) for G in GS if G <= 8]   # (|g|, probe mode)
+
+
+@pytest.mark.parametrize("G,mode", MODES)
+def test_config1_unique_parity(wd, G, mode):
     # BASELINE config 1: 2^20 unique keys, load 0.95, all keys + 2^20 absent keys queried
     n, ks, vs = 1 << 20, 101, 202
     keys, vals = wdgen.unique_keys(n, ks), wdgen.values(n, vs)
     q = wdgen.interleaved_queries(n, ks)
     with wd.Table(capacity_for(n, 0.95), 1, G) as t:
+        t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0
         assert t.size() == n
@@ -50,13 +54,15 @@ def test_config1_unique_parity(wd, G):
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
 
 
+@pytest.mark.parametrize("mode", [0, 1])
 @pytest.mark.parametrize("kif", [4, 8])
 @pytest.mark.parametrize("alpha", [0.8, 0.99, 0.999])
-def test_alpha_and_keys_in_flight(wd, alpha, kif):
+def test_alpha_and_keys_in_flight(wd, alpha, kif, mode):
     n = 300_001  # ragged
     keys, vals = wdgen.unique_keys(n, 7), wdgen.values(n, 8)
     q = wdgen.interleaved_queries(n, 7)
     with wd.Table(capacity_for(n, alpha), 1, 4) as t:
+        t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, kif)
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0 and t.size() == n
@@ -64,8 +70,8 @@ def test_alpha_and_keys_in_flight(wd, alpha, kif):
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
 
 
-@pytest.mark.parametrize("G", GS)
-def test_serial_layout_equals_fig3_replay(wd, G):
+@pytest.mark.parametrize("G,mode", MODES)
+def test_serial_layout_equals_fig3_replay(wd, G, mode):
     # WD_OPT_SERIAL runs one probing group, one key at a time: the slot layout must equal
     # the oracle's sequential replay of Fig. 3 bit for bit (probe sequence, windows,
     # leftmost-empty leader, update-on-match).
@@ -77,6 +83,7 @@ def test_serial_layout_equals_fig3_replay(wd, G):
     r.insert(keys, vals)
     with wd.Table(3200, 1, G) as t:
         assert t.shard_capacity() == c
+        t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_SERIAL, 1)
         t.insert(to_dev(keys), to_dev(vals))
         assert t.sync() == 0
@@ -85,30 +92,34 @@ def test_serial_layout_equals_fig3_replay(wd, G):
     assert np.array_equal(slots, r.table)
 
 
-@pytest.mark.parametrize("Gi,Gq", [(1, 32), (32, 1), (4, 8), (8, 2), (2, 16)])
-def test_cross_group_size(wd, Gi, Gq):
+@pytest.mark.parametrize("Gi,Gq,mi,mq", [(1, 32, 0, 0), (32, 1, 0, 1), (4, 8, 1, 0),
+                                         (8, 2, 0, 1), (2, 16, 1, 0), (4, 4, 1, 0), (4, 4, 0, 1)])
+def test_cross_group_size(wd, Gi, Gq, mi, mq):
     # the probing scheme is consistent when |g| varies: insert with one |g|, query
-    # with another.
+    # with another — and across the two probe modes (same windows, same sequence).
     n = 200_000
     keys, vals = wdgen.unique_keys(n, 9), wdgen.values(n, 9)
     q = wdgen.interleaved_queries(n, 9)
     with wd.Table(capacity_for(n, 0.97), 1, Gi) as t:
+        t.set_option(wd.WD_OPT_PROBE_MODE, mi)
         t.insert(to_dev(keys), to_dev(vals))
         t.set_option(wd.WD_OPT_GROUP_SIZE, Gq)
+        t.set_option(wd.WD_OPT_PROBE_MODE, mq)
         ov, of = t.retrieve(to_dev(q))
         gv, gf = from_dev(ov), of.cpu().numpy()
     cv, cf = oracle.expected_unique(q, n, 9, 9)
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
 
 
-@pytest.mark.parametrize("G", [1, 4, 32])
-def test_duplicates_upsert(wd, G):
+@pytest.mark.parametrize("G,mode", [(1, 0), (4, 0), (32, 0), (2, 1), (4, 1), (8, 1)])
+def test_duplicates_upsert(wd, G, mode):
     # duplicate-key mode: value must be one of the values inserted for the key;
     # size = number of distinct keys; a second stream-ordered call wins.
     n = 400_000
     keys = wdgen.uniform_keys(n, 11) % np.uint32(150_000)
     vals = wdgen.values(n, 12)
     with wd.Table(capacity_for(150_000, 0.9), 1, G) as t:
+        t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.insert(to_dev(keys), to_dev(vals))
         q = np.arange(160_000, dtype=np.uint32)
         ov, of = t.retrieve(to_dev(q))

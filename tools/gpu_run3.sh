@@ -1,7 +1,7 @@
 timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1
 rm -f gpurun_out/kg.txt
 for k in 4 8; do for g in 1 2 4 8 16 32; do
-  timeout 120 python bench.py --steps 5 --warmup 2 --no-e2e --no-cpu --kif $k --group-size $g 2>&1 | python -c "import json,sys; d=json.loads(sys.stdin.read().strip().splitlines()[-1]); print('K=$k G=$g', round(d['insert_gops'],2), round(d['query_gops'],2), round(d['roofline']['frac'],3), round(d['roofline']['other']['frac'],3))" >> gpurun_out/kg.txt 2>&1
+  timeout 120 python bench.py --steps 5 --warmup 2 --no-e2e --no-cpu --kif $k --group-size $g $EXTRA 2>&1 | python -c "import json,sys; d=json.loads(sys.stdin.read().strip().splitlines()[-1]); print('K=$k G=$g', round(d['insert_gops'],2), round(d['query_gops'],2), round(d['roofline']['frac'],3), round(d['roofline']['other']['frac'],3))" >> gpurun_out/kg.txt 2>&1
 done; done
 bash tools/gpu_prof.sh k4c
 echo done

@@ -50,6 +50,57 @@ __global__ void __launch_bounds__(256) gather(unsigned long long* buf, uint64_t 
   if (acc == 42) sink[0] = acc;
 }
 
+// dependent chains: each lane follows D independent chains; the next window of a chain is
+// derived from the data just loaded (as in probing), so only D windows per lane are ever
+// in flight.  WB = window bytes loaded by ONE lane with vector loads (8/16/32).
+template <int D, int WB>
+__global__ void __launch_bounds__(256) chase(unsigned long long* buf, uint64_t nwin, int iters,
+                                             unsigned long long* sink) {
+  const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t cur[D];
+  unsigned long long acc = 0;
+#pragma unroll
+  for (int d = 0; d < D; ++d) cur[d] = hash32(tid * 2654435761u + d * 97u + 5u);
+  for (int it = 0; it < iters; ++it) {
+    unsigned long long v[D];
+#pragma unroll
+    for (int d = 0; d < D; ++d) {
+      const uint64_t w = (uint64_t(cur[d]) * nwin) >> 32;
+      const unsigned long long* p = buf + w * 4;
+      if (WB == 32) {
+        unsigned long long a, b, c, e;
+        asm volatile("ld.global.cg.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(a), "=l"(b), "=l"(c), "=l"(e) : "l"(p));
+        v[d] = a ^ b ^ c ^ e;
+      } else {
+        v[d] = ldr(p);
+      }
+    }
+#pragma unroll
+    for (int d = 0; d < D; ++d) {
+      acc += v[d];
+      cur[d] = hash32(cur[d] ^ uint32_t(v[d]) ^ uint32_t(it));   // next address depends on data
+    }
+  }
+  if (acc == 42) sink[0] = acc;
+}
+
+template <int D, int WB>
+void run_chase(unsigned long long* buf, uint64_t bytes, int grid, int iters, unsigned long long* sink,
+               const char* tag) {
+  const uint64_t nwin = (bytes - 256) / 32;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a); cudaEventCreate(&b);
+  chase<D, WB><<<grid, 256>>>(buf, nwin, 2, sink);
+  cudaEventRecord(a);
+  chase<D, WB><<<grid, 256>>>(buf, nwin, iters, sink);
+  cudaEventRecord(b);
+  cudaEventSynchronize(b);
+  float ms; cudaEventElapsedTime(&ms, a, b);
+  const double windows = double(grid) * 256 * D * iters;
+  printf("%.2fGB chase W=%2dB D=%d %s: %6.1f Gwin/s  (%d thr/SM x %d chains)\n", bytes / 1e9, WB, D, tag,
+         windows / (ms * 1e-3) / 1e9, grid * 256 / 148, D);
+}
+
 template <int D, int MODE, int WB, int AB>
 void run(const char* name, unsigned long long* buf, uint64_t bytes, int grid, int iters,
          unsigned long long* sink) {
@@ -91,6 +142,13 @@ int main() {
     run<8, 2, 32, 32>("casw", buf, bytes, grid, it, sink);
     run<8, 1, 64, 64>("cas", buf, bytes, grid, it, sink);
     run<8, 2, 64, 64>("casw", buf, bytes, grid, it, sink);
+    for (int occ : {2, 4, 8}) {
+      run_chase<1, 32>(buf, bytes, sms * occ, 64, sink, "");
+      run_chase<2, 32>(buf, bytes, sms * occ, 64, sink, "");
+      run_chase<4, 32>(buf, bytes, sms * occ, 64, sink, "");
+      run_chase<8, 32>(buf, bytes, sms * occ, 32, sink, "");
+      run_chase<4, 8>(buf, bytes, sms * occ, 64, sink, "");
+    }
     cudaFree(buf);
   }
   printf("err: %s\n", cudaGetErrorString(cudaGetLastError()));
