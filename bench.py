@@ -52,7 +52,7 @@ def parse():
     ap.add_argument("--group-size", type=int, default=4)
     ap.add_argument("--kif", type=int, default=0, help="keys in flight per group (0=default)")
     ap.add_argument("--probe-mode", type=int, default=None,
-                    help="0: cooperative group per window (Fig. 3); 1: lane-window")
+                    help="0: auto; 1: cooperative group per window (Fig. 3); 2: lane-window")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--dist-backend", default="nccl",

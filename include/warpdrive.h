@@ -142,8 +142,10 @@ typedef enum {
     WD_OPT_KEYS_IN_FLIGHT = 4, /* 0 = default; else keys per group in flight (4 or 8) */
     WD_OPT_PART_SEED = 5,    /* seed of the partition function p(k) (C15) */
     WD_OPT_PART_MODE = 6,    /* 0: p(k) = fmix32(k+seed)*m >> 32; 1: k mod m (Fig. 4) */
-    WD_OPT_PROBE_MODE = 7,   /* 0: cooperative group of |g| lanes per window (Fig. 3);
-                                1: lane-window — one lane loads the whole |g|-slot window with
+    WD_OPT_PROBE_MODE = 7,   /* 0 (default): auto — lane-window when the shard fits in half
+                                the L2 (<= 64 MB) and |g| <= 8, else cooperative group;
+                                1: cooperative group of |g| lanes per window (Fig. 3);
+                                2: lane-window — one lane loads the whole |g|-slot window with
                                 one sm_100 vector load (|g| <= 8; same windows, same result) */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */

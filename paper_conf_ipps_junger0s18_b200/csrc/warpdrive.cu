@@ -116,7 +116,7 @@ struct wd_table {
   int G = 4;
   int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit
   int kif = 0;        // keys in flight per group (0 = default)
-  int probe_mode = 0; // 0: cooperative groups (Fig. 3), 1: lane-window (|g| <= 8)
+  int probe_mode = 0; // 0: auto, 1: cooperative groups (Fig. 3), 2: lane-window (|g| <= 8)
   uint64_t batch = 1ull << 24;
   int serial = 0;
   uint32_t pseed = 0x9E3779B9u;
@@ -228,7 +228,12 @@ template <int G, bool INSERT, class In, class Out>
 wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
   if constexpr (G <= 8) {
-    if (t->probe_mode == 1) {
+    // auto: the lane-window kernel issues 32/|g| x fewer instructions per window and wins
+    // when the table is L2-resident (measured 2-4x); from HBM the cooperative-group kernel
+    // keeps the tail of each warp step shorter (max over 32/|g| loads, not 32) and wins.
+    const bool lane = t->probe_mode == 2 ||
+                      (t->probe_mode == 0 && s.cap * sizeof(unsigned long long) <= (64ull << 20));
+    if (lane) {
       const int k = lane_k(G, t->kif);
       if (k == 1) return launch_lane_k<G, 1, INSERT>(t, s, in, out, n_hint, st);
       if (k == 2) return launch_lane_k<G, 2, INSERT>(t, s, in, out, n_hint, st);
@@ -1113,7 +1118,7 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       return WD_OK;
     case WD_OPT_PART_SEED: t->pseed = uint32_t(v); return WD_OK;
     case WD_OPT_PROBE_MODE:
-      if (v != 0 && v != 1) return fail(WD_ERR_INVALID_ARG, "probe mode %lld", (long long)v);
+      if (v < 0 || v > 2) return fail(WD_ERR_INVALID_ARG, "probe mode %lld", (long long)v);
       t->probe_mode = int(v);
       return WD_OK;
     case WD_OPT_PART_MODE:

@@ -23,7 +23,7 @@ def wd():
 
 
 @pytest.mark.parametrize("m", [2, 3, 4, 8])
-@pytest.mark.parametrize("G,mode", [(1, 0), (4, 0), (32, 0), (4, 1)])
+@pytest.mark.parametrize("G,mode", [(1, 1), (4, 1), (32, 1), (4, 2), (4, 0)])
 def test_loopback_unique_parity(wd, m, G, mode):
     n = 200_000 + 17 * m
     keys, vals = wdgen.unique_keys(n, 21), wdgen.values(n, 22)

@@ -27,7 +27,7 @@ def _oracle_answers(keys, vals, queries, dup=False):
     return m, *m.retrieve(queries)
 
 
-MODES = [(G, 0) for G in GS] + [(G, 1) for G in GS if G <= 8]   # (|g|, probe mode)
+MODES = [(G, 1) for G in GS] + [(G, 2) for G in GS if G <= 8]   # (|g|, probe mode)
 
 
 @pytest.mark.parametrize("G,mode", MODES)
@@ -54,7 +54,7 @@ def test_config1_unique_parity(wd, G, mode):
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
 
 
-@pytest.mark.parametrize("mode", [0, 1])
+@pytest.mark.parametrize("mode", [1, 2])
 @pytest.mark.parametrize("kif", [4, 8])
 @pytest.mark.parametrize("alpha", [0.8, 0.99, 0.999])
 def test_alpha_and_keys_in_flight(wd, alpha, kif, mode):
@@ -92,8 +92,8 @@ def test_serial_layout_equals_fig3_replay(wd, G, mode):
     assert np.array_equal(slots, r.table)
 
 
-@pytest.mark.parametrize("Gi,Gq,mi,mq", [(1, 32, 0, 0), (32, 1, 0, 1), (4, 8, 1, 0),
-                                         (8, 2, 0, 1), (2, 16, 1, 0), (4, 4, 1, 0), (4, 4, 0, 1)])
+@pytest.mark.parametrize("Gi,Gq,mi,mq", [(1, 32, 1, 1), (32, 1, 1, 2), (4, 8, 2, 1),
+                                         (8, 2, 1, 2), (2, 16, 2, 0), (4, 4, 2, 1), (4, 4, 1, 2)])
 def test_cross_group_size(wd, Gi, Gq, mi, mq):
     # the probing scheme is consistent when |g| varies: insert with one |g|, query
     # with another — and across the two probe modes (same windows, same sequence).
@@ -111,7 +111,7 @@ def test_cross_group_size(wd, Gi, Gq, mi, mq):
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
 
 
-@pytest.mark.parametrize("G,mode", [(1, 0), (4, 0), (32, 0), (2, 1), (4, 1), (8, 1)])
+@pytest.mark.parametrize("G,mode", [(1, 1), (4, 1), (32, 1), (2, 2), (4, 2), (8, 2), (4, 0)])
 def test_duplicates_upsert(wd, G, mode):
     # duplicate-key mode: value must be one of the values inserted for the key;
     # size = number of distinct keys; a second stream-ordered call wins.

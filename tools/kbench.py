@@ -37,14 +37,14 @@ def rate(n, G, mode, alpha=0.95, kif=0, reps=5):
 if __name__ == "__main__" and (len(sys.argv) < 2 or sys.argv[1] != "noout"):
     if len(sys.argv) > 1 and sys.argv[1] == "k":
         lg = int(sys.argv[2]) if len(sys.argv) > 2 else 28
-        for G, m, ks in [(4, 0, (2, 4, 8)), (4, 1, (1, 2, 4, 8)), (8, 1, (1, 2, 4)),
-                         (2, 1, (2, 4, 8)), (8, 0, (2, 4, 8)), (1, 1, (2, 4, 8))]:
+        for G, m, ks in [(4, 1, (2, 4, 8)), (4, 2, (1, 2, 4, 8)), (8, 2, (1, 2, 4)),
+                         (2, 2, (2, 4, 8)), (8, 1, (2, 4, 8)), (1, 2, (2, 4, 8))]:
             for k in ks:
                 i, q = rate(1 << lg, G, m, kif=k)
                 print(f"n=2^{lg} G={G} mode={m} K={k}: insert {i:6.2f} G/s  query {q:6.2f} G/s",
                       flush=True)
         sys.exit(0)
-    cfgs = [(G, m) for m in (0, 1) for G in (2, 4, 8)]
+    cfgs = [(G, m) for m in (1, 2) for G in (2, 4, 8)]
     for lg in (20, 22, 24, 26, 28):
         for G, m in cfgs:
             i, q = rate(1 << lg, G, m)
@@ -74,6 +74,6 @@ def query_no_out(n, G, mode, kif=0, alpha=0.95, reps=5):
 
 
 if __name__ == "__main__" and len(sys.argv) > 1 and sys.argv[1] == "noout":
-    for G, m, k in [(4, 0, 8), (4, 1, 4), (4, 1, 1), (8, 0, 4), (8, 1, 2), (1, 1, 8)]:
+    for G, m, k in [(4, 1, 8), (4, 2, 4), (4, 2, 1), (8, 1, 4), (8, 2, 2), (1, 2, 8)]:
         print(f"G={G} mode={m} K={k}: query without outputs {query_no_out(1 << 28, G, m, k):6.2f} G/s; "
               f"with: {rate(1 << 28, G, m, kif=k)[1]:6.2f} G/s", flush=True)

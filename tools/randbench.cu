@@ -101,6 +101,75 @@ void run_chase(unsigned long long* buf, uint64_t bytes, int grid, int iters, uns
          windows / (ms * 1e-3) / 1e9, grid * 256 / 148, D);
 }
 
+// chase2: probe-like chains.  Each chain works on "keys": a key starts at a random
+// 32-B-aligned window and continues with the ADJACENT window with probability ~1/2 (so
+// ~2 windows per key, like alpha = 0.95, |g| = 4).  Variants add the probe kernel's other
+// traffic: V&1: read a 4-byte input key per key (sequential per lane); V&2: write a 4-byte
+// + 1-byte output per key (scattered by key index); V&4: CAS the last window (insert-like,
+// succeeds -> dirty line).
+template <int D, int V>
+__global__ void __launch_bounds__(256) chase2(unsigned long long* buf, uint64_t nwin, int keys_per_chain,
+                                              const uint32_t* in, uint32_t* out_v, uint8_t* out_f,
+                                              unsigned long long* sink) {
+  const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t nthr = gridDim.x * blockDim.x;
+  uint32_t cur[D], kidx[D];
+  uint64_t w[D];
+  unsigned long long acc = 0;
+#pragma unroll
+  for (int d = 0; d < D; ++d) {
+    kidx[d] = 0;
+    cur[d] = hash32(tid * 2654435761u + d * 97u + 5u);
+    w[d] = (uint64_t(cur[d]) * nwin) >> 32;
+  }
+  int done_keys = 0;
+  const int total = keys_per_chain * D;
+  while (done_keys < total) {
+    unsigned long long v[D];
+#pragma unroll
+    for (int d = 0; d < D; ++d) {
+      const unsigned long long* p = buf + w[d] * 4;
+      unsigned long long a, b, c, e;
+      asm volatile("ld.global.cg.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(a), "=l"(b), "=l"(c), "=l"(e) : "l"(p));
+      v[d] = a ^ b ^ c ^ e;
+    }
+#pragma unroll
+    for (int d = 0; d < D; ++d) {
+      acc += v[d];
+      cur[d] = hash32(cur[d] ^ uint32_t(v[d]) ^ 0x9e37u);
+      const bool cont = (cur[d] & 1u) && w[d] + 1 < nwin;          // adjacent next window
+      if (cont) { w[d] += 1; continue; }
+      // key finished
+      const uint64_t item = uint64_t(kidx[d]) * nthr * D + uint64_t(tid) * D + d;
+      if (V & 4) acc += atomicCAS(buf + w[d] * 4, v[d], v[d] ^ 1ull);
+      if (V & 2) { out_v[item] = uint32_t(v[d]); out_f[item] = 1; }
+      ++kidx[d];
+      ++done_keys;
+      uint32_t nk = cur[d];
+      if (V & 1) nk ^= __ldg(in + item);
+      w[d] = (uint64_t(hash32(nk)) * nwin) >> 32;
+    }
+  }
+  if (acc == 42) sink[0] = acc;
+}
+
+template <int D, int V>
+void run_chase2(unsigned long long* buf, uint64_t bytes, int grid, int kpc, uint32_t* in, uint32_t* ov,
+                uint8_t* of, unsigned long long* sink) {
+  const uint64_t nwin = (bytes - 256) / 32;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a); cudaEventCreate(&b);
+  chase2<D, V><<<grid, 256>>>(buf, nwin, 2, in, ov, of, sink);
+  cudaEventRecord(a);
+  chase2<D, V><<<grid, 256>>>(buf, nwin, kpc, in, ov, of, sink);
+  cudaEventRecord(b);
+  cudaEventSynchronize(b);
+  float ms; cudaEventElapsedTime(&ms, a, b);
+  const double keys = double(grid) * 256 * D * kpc;
+  printf("%.2fGB chase2 V=%d D=%d (%d thr/SM): %6.2f G keys/s  (~%.1f G windows/s)\n", bytes / 1e9, V, D,
+         grid * 256 / 148, keys / (ms * 1e-3) / 1e9, 2 * keys / (ms * 1e-3) / 1e9);
+}
+
 template <int D, int MODE, int WB, int AB>
 void run(const char* name, unsigned long long* buf, uint64_t bytes, int grid, int iters,
          unsigned long long* sink) {
@@ -142,6 +211,23 @@ int main() {
     run<8, 2, 32, 32>("casw", buf, bytes, grid, it, sink);
     run<8, 1, 64, 64>("cas", buf, bytes, grid, it, sink);
     run<8, 2, 64, 64>("casw", buf, bytes, grid, it, sink);
+    {
+      const int grid = sms * 4, kpc = 32;
+      const size_t nk = size_t(grid) * 256 * 8 * kpc;
+      uint32_t *in, *ov; uint8_t* of;
+      cudaMalloc(&in, nk * 4); cudaMalloc(&ov, nk * 4); cudaMalloc(&of, nk);
+      cudaMemset(in, 1, nk * 4);
+      run_chase2<4, 0>(buf, bytes, grid, kpc, in, ov, of, sink);
+      run_chase2<4, 1>(buf, bytes, grid, kpc, in, ov, of, sink);
+      run_chase2<4, 2>(buf, bytes, grid, kpc, in, ov, of, sink);
+      run_chase2<4, 3>(buf, bytes, grid, kpc, in, ov, of, sink);
+      run_chase2<4, 4>(buf, bytes, grid, kpc, in, ov, of, sink);
+      run_chase2<4, 7>(buf, bytes, grid, kpc, in, ov, of, sink);
+      run_chase2<8, 0>(buf, bytes, grid, kpc / 2, in, ov, of, sink);
+      run_chase2<8, 3>(buf, bytes, grid, kpc / 2, in, ov, of, sink);
+      cudaMemset(buf, 0xff, bytes);
+      cudaFree(in); cudaFree(ov); cudaFree(of);
+    }
     for (int occ : {2, 4, 8}) {
       run_chase<1, 32>(buf, bytes, sms * occ, 64, sink, "");
       run_chase<2, 32>(buf, bytes, sms * occ, 64, sink, "");
