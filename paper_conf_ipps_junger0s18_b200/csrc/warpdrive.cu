@@ -88,6 +88,7 @@ struct Shard {
   unsigned long long* slots = nullptr;
   unsigned long long* counters = nullptr;
   cudaStream_t s_main = nullptr, s_h2d = nullptr, s_d2h = nullptr;
+  cudaStream_t s_probe = nullptr;   // phase B of the cascade (own stream unless loopback)
   bool own_main = true;
   // exchange arena (one allocation: IPC-exportable)
   void* arena = nullptr;
@@ -104,6 +105,7 @@ struct Shard {
   uint8_t* pin_fout[2] = {};
   cudaEvent_t ev_h2d[2] = {}, ev_free[2] = {}, ev_kdone[2] = {}, ev_d2h[2] = {};
   cudaEvent_t ev_join_main = nullptr, ev_join_h2d = nullptr, ev_join_d2h = nullptr;
+  cudaEvent_t ev_join_probe = nullptr;
   bool h2d_pending[2] = {false, false}, d2h_pending[2] = {false, false};
 };
 
@@ -285,10 +287,11 @@ wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
   CK(cudaMalloc(&s.slots, cap * sizeof(unsigned long long)));
   CK(cudaMalloc(&s.counters, wd::CNT_N * sizeof(unsigned long long)));
   if (shared_main) {
-    s.s_main = shared_main;
+    s.s_main = s.s_probe = shared_main;   // loopback: one stream, phases in issue order
     s.own_main = false;
   } else {
     CK(cudaStreamCreateWithFlags(&s.s_main, cudaStreamNonBlocking));
+    CK(cudaStreamCreateWithFlags(&s.s_probe, cudaStreamNonBlocking));
   }
   CK(cudaStreamCreateWithFlags(&s.s_h2d, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&s.s_d2h, cudaStreamNonBlocking));
@@ -301,6 +304,7 @@ wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
   CK(cudaEventCreateWithFlags(&s.ev_join_main, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&s.ev_join_h2d, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&s.ev_join_d2h, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&s.ev_join_probe, cudaEventDisableTiming));
   // a1: fresh table
   const int grid = t->sm_count * 4;
   wd::fill_kernel<<<grid, wd::kBlock, 0, s.s_main>>>(s.slots, s.cap, s.counters, wd::CNT_N);
@@ -345,6 +349,7 @@ void free_staging(Shard& s) {
 void shard_free(Shard& s) {
   DeviceGuard g(s.device);
   if (s.s_main) cudaStreamSynchronize(s.s_main);
+  if (s.s_probe) cudaStreamSynchronize(s.s_probe);
   if (s.s_h2d) cudaStreamSynchronize(s.s_h2d);
   if (s.s_d2h) cudaStreamSynchronize(s.s_d2h);
   free_exchange(s);
@@ -360,7 +365,9 @@ void shard_free(Shard& s) {
   if (s.ev_join_main) cudaEventDestroy(s.ev_join_main);
   if (s.ev_join_h2d) cudaEventDestroy(s.ev_join_h2d);
   if (s.ev_join_d2h) cudaEventDestroy(s.ev_join_d2h);
+  if (s.ev_join_probe) cudaEventDestroy(s.ev_join_probe);
   if (s.own_main && s.s_main) cudaStreamDestroy(s.s_main);
+  if (s.own_main && s.s_probe) cudaStreamDestroy(s.s_probe);
   if (s.s_h2d) cudaStreamDestroy(s.s_h2d);
   if (s.s_d2h) cudaStreamDestroy(s.s_d2h);
   s = Shard{};
@@ -443,6 +450,7 @@ wd_status_t ensure_exchange(wd_table* t) {
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
     CK(cudaStreamSynchronize(s.s_main));
+    CK(cudaStreamSynchronize(s.s_probe));
   }
   for (void* p : t->opened) cudaIpcCloseMemHandle(p);
   t->opened.clear();
@@ -487,6 +495,7 @@ wd_status_t fork_from(wd_table* t, cudaStream_t stream, cudaEvent_t* ev_tmp) {
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
     CK(cudaStreamWaitEvent(s.s_main, *ev_tmp, 0));
+    if (s.s_probe != s.s_main) CK(cudaStreamWaitEvent(s.s_probe, *ev_tmp, 0));
     CK(cudaStreamWaitEvent(s.s_h2d, *ev_tmp, 0));
     CK(cudaStreamWaitEvent(s.s_d2h, *ev_tmp, 0));
   }
@@ -497,6 +506,10 @@ wd_status_t join_into(wd_table* t, cudaStream_t stream, cudaEvent_t ev_tmp) {
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
     CK(cudaEventRecord(s.ev_join_main, s.s_main));
+    if (s.s_probe != s.s_main) {
+      CK(cudaEventRecord(s.ev_join_probe, s.s_probe));
+      CK(cudaStreamWaitEvent(stream, s.ev_join_probe, 0));
+    }
     CK(cudaEventRecord(s.ev_join_h2d, s.s_h2d));
     CK(cudaEventRecord(s.ev_join_d2h, s.s_d2h));
     CK(cudaStreamWaitEvent(stream, s.ev_join_main, 0));
@@ -629,15 +642,15 @@ wd::FlagPtrs flag_ptrs(wd_table* t, int flag, int who) {
   return f;
 }
 
-wd_status_t launch_wait(wd_table* t, Shard& s, int flag, unsigned long long target) {
-  wd::wait_kernel<<<1, 32, 0, s.s_main>>>(s.self.flags + flag * t->m, t->m, target,
-                                          kWaitTimeoutNs, s.counters);
+wd_status_t launch_wait(wd_table* t, Shard& s, cudaStream_t st, int flag, unsigned long long target) {
+  wd::wait_kernel<<<1, 32, 0, st>>>(s.self.flags + flag * t->m, t->m, target, kWaitTimeoutNs,
+                                    s.counters);
   CK(cudaGetLastError());
   t->launches++;
   return WD_OK;
 }
-wd_status_t launch_signal(wd_table* t, Shard& s, int flag, unsigned long long epoch) {
-  wd::signal_kernel<<<1, 32, 0, s.s_main>>>(flag_ptrs(t, flag, s.id), t->m, epoch);
+wd_status_t launch_signal(wd_table* t, Shard& s, cudaStream_t st, int flag, unsigned long long epoch) {
+  wd::signal_kernel<<<1, 32, 0, st>>>(flag_ptrs(t, flag, s.id), t->m, epoch);
   CK(cudaGetLastError());
   t->launches++;
   return WD_OK;
@@ -668,10 +681,18 @@ wd_status_t cascade_op(wd_table* t, bool insert, std::vector<IO>& ios, cudaStrea
   TRY(fork_from(t, stream, &ev0));
   for (auto& s : t->local) s.h2d_pending[0] = s.h2d_pending[1] = false;
 
-  for (uint64_t b = 0; b < nbt; ++b) {
-    const unsigned long long e = t->epoch + 1 + b;
+  // Three phases per batch b (epoch e = epoch0 + 1 + b, exchange slot e % 2):
+  //   A (s_main):  multisplit fused with the push into the owners' receive regions, then
+  //                publish the row of T and the READY flags
+  //   B (s_probe): wait for the column of T, probe (insert / retrieve), DONE flags
+  //   C (s_main):  queries only — pull the results back, unpermute, RESC flags
+  // Issued as A(0), then A(b+1), B(b), C(b): the multisplit and transposition of batch b+1
+  // overlap the probing of batch b (Fig. 5's MST || INS), and the query's reverse pull of
+  // batch b never blocks the next multisplit.  Cross-shard ordering is by epoch flags only.
+  const unsigned long long e0 = t->epoch;
+  auto phaseA = [&](uint64_t b) -> wd_status_t {
+    const unsigned long long e = e0 + 1 + b;
     const int slot = int(e & 1);
-    // ---- phase A: every local shard multisplits its batch into the owners' regions
     for (size_t r = 0; r < t->local.size(); ++r) {
       Shard& s = t->local[r];
       const IO& io = ios[r];
@@ -679,7 +700,7 @@ wd_status_t cascade_op(wd_table* t, bool insert, std::vector<IO>& ios, cudaStrea
       const uint64_t off = std::min(io.n, b * B), cnt = std::min(B, io.n - off);
       const uint32_t *dk = nullptr, *dv = nullptr;
       TRY(stage_in(s, io, off, cnt, int(b & 1), insert, &dk, &dv));
-      if (e > 2) TRY(launch_wait(t, s, FLAG_DONE, e - 2));  // owners released region e-2
+      if (e > 2) TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e - 2));  // owners released e-2
       if (cnt) {
         wd::DstPtrs dst{};
         for (int d = 0; d < m; ++d) {
@@ -706,30 +727,37 @@ wd_status_t cascade_op(wd_table* t, bool insert, std::vector<IO>& ios, cudaStrea
       CK(cudaGetLastError());
       t->launches++;
     }
-    // ---- phase B: every local shard inserts / queries its column of T
+    return WD_OK;
+  };
+  auto phaseB = [&](uint64_t b) -> wd_status_t {
+    const unsigned long long e = e0 + 1 + b;
+    const int slot = int(e & 1);
     for (auto& s : t->local) {
       DeviceGuard g(s.device);
-      TRY(launch_wait(t, s, FLAG_READY, e));
+      TRY(launch_wait(t, s, s.s_probe, FLAG_READY, e));
       if (insert) {
         const wd::InSeg<true> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
-        TRY(launch_probe<true>(t, s, in, wd::OutNone{}, B, s.s_main));
+        TRY(launch_probe<true>(t, s, in, wd::OutNone{}, B, s.s_probe));
       } else {
         // origins consumed the results of the previous query epoch that used this slot
-        if (t->res_used[slot]) TRY(launch_wait(t, s, FLAG_RESC, t->res_used[slot]));
+        if (t->res_used[slot]) TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
         const wd::InSeg<false> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
-        TRY(launch_probe<false>(t, s, in, wd::OutPacked{s.self.res[slot]}, B, s.s_main));
+        TRY(launch_probe<false>(t, s, in, wd::OutPacked{s.self.res[slot]}, B, s.s_probe));
       }
-      TRY(launch_signal(t, s, FLAG_DONE, e));
+      TRY(launch_signal(t, s, s.s_probe, FLAG_DONE, e));
     }
-    if (insert) continue;
-    t->res_used[slot] = e;
-    // ---- phase C (query): every origin pulls its results back and unpermutes
+    if (!insert) t->res_used[slot] = e;
+    return WD_OK;
+  };
+  auto phaseC = [&](uint64_t b) -> wd_status_t {
+    const unsigned long long e = e0 + 1 + b;
+    const int slot = int(e & 1);
     for (size_t r = 0; r < t->local.size(); ++r) {
       Shard& s = t->local[r];
       const IO& io = ios[r];
       DeviceGuard g(s.device);
       const uint64_t off = std::min(io.n, b * B), cnt = std::min(B, io.n - off);
-      TRY(launch_wait(t, s, FLAG_DONE, e));
+      TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e));
       if (cnt) {
         wd::DstPtrs src{};
         for (int d = 0; d < m; ++d) src.p[d] = t->peers[d].res[slot] + uint64_t(s.id) * B;
@@ -741,9 +769,17 @@ wd_status_t cascade_op(wd_table* t, bool insert, std::vector<IO>& ios, cudaStrea
         CK(cudaGetLastError());
         t->launches++;
       }
-      TRY(launch_signal(t, s, FLAG_RESC, e));
+      TRY(launch_signal(t, s, s.s_main, FLAG_RESC, e));
       TRY(stage_out(s, io, off, cnt, int(b & 1), true));
     }
+    return WD_OK;
+  };
+
+  TRY(phaseA(0));
+  for (uint64_t b = 0; b < nbt; ++b) {
+    if (b + 1 < nbt) TRY(phaseA(b + 1));
+    TRY(phaseB(b));
+    if (!insert) TRY(phaseC(b));
   }
   t->epoch += nbt;
   return join_into(t, stream, ev0);
@@ -855,6 +891,7 @@ wd_status_t sticky_status(wd_table* t) {
     DeviceGuard g(s.device);
     unsigned long long c[wd::CNT_N];
     CK(cudaStreamSynchronize(s.s_main));
+    CK(cudaStreamSynchronize(s.s_probe));
     CK(cudaStreamSynchronize(s.s_h2d));
     CK(cudaStreamSynchronize(s.s_d2h));
     CK(cudaDeviceSynchronize());
