@@ -412,6 +412,44 @@ def run_sweep(args, wd, gg, torch):
                             "insert_gops": n / ims / 1e6, "query_gops": n / qms / 1e6,
                             "insert_frac": n * (40 + 32 * pc["ins_sectors"]) / (ims * 1e-3) / 1e9 / hbm,
                             "query_frac": n * (9 + 32 * pc["hit_sectors"]) / (qms * 1e-3) / 1e9 / hbm})
+    del keys, vals, vout, fout
+    out += run_zipf(wd, gg, torch)
+    return out
+
+
+def run_zipf(wd, gg, torch, log2n=27):
+    """SURVEY §8(f) #1 / Fig. 8 protocol: 2^27 Zipf(s = 1 + 1e-6) draws over
+    the 4-byte key space, insert all then retrieve all; load = actual occupancy (distinct
+    keys / capacity).  Extra lines, not the headline."""
+    out = []
+    n = 1 << log2n
+    keys = gg.zipf_keys(n, 2**32 - 1, KEY_SEED)
+    vals = gg.values(n, VAL_SEED)
+    distinct = int(torch.unique(keys).numel())
+    vout = torch.empty(n, dtype=torch.int32, device="cuda")
+    fout = torch.empty(n, dtype=torch.uint8, device="cuda")
+    s = torch.cuda.current_stream()
+    for alpha in (0.8, 0.95):
+        for G in (1, 2, 4, 8, 16):
+            with wd.Table(int(math.ceil(distinct / alpha)), 1, G) as t:
+                ti, tq = [], []
+                for it in range(4):
+                    a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+                    t.clear(s)
+                    a.record(s)
+                    t.insert(keys, vals, s)
+                    b.record(s)
+                    t.retrieve(keys, vout, fout, s)
+                    c.record(s)
+                    torch.cuda.synchronize()
+                    if it:
+                        ti.append(a.elapsed_time(b))
+                        tq.append(b.elapsed_time(c))
+                assert t.sync() == 0 and t.size() == distinct
+                assert bool((fout == 1).all())
+                ims, qms = sum(ti) / len(ti), sum(tq) / len(tq)
+                out.append({"sweep": "zipf", "draws": n, "distinct": distinct, "alpha": alpha,
+                            "G": G, "insert_gops": n / ims / 1e6, "query_gops": n / qms / 1e6})
     return out
 
 

@@ -147,6 +147,9 @@ typedef enum {
                                 1: cooperative group of |g| lanes per window (Fig. 3);
                                 2: lane-window — one lane loads the whole |g|-slot window with
                                 one sm_100 vector load (|g| <= 8; same windows, same result) */
+    WD_OPT_KERNEL_FLAGS = 8, /* bit 0: probe loads may hit L1 (safe: keys never change once
+                                written; a lost CAS reloads from L2); bit 1: value updates
+                                of existing keys as atomic exchange.  Default 3. */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -119,6 +119,10 @@ struct wd_table {
   int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit
   int kif = 0;        // keys in flight per group (0 = default)
   int probe_mode = 0; // 0: auto, 1: cooperative groups (Fig. 3), 2: lane-window (|g| <= 8)
+  // wd::kF_* kernel variants (WD_OPT_KERNEL_FLAGS).  Default both: atom.exch value updates
+  // take hot (Zipf) keys from 0.5 to 6-8 G inserts/s (tools/flags_bench.py), L1-allowed
+  // probe loads add ~15 % there; neither changes the unique-key rates.
+  uint32_t kflags = wd::kF_L1 | wd::kF_XCHG;
   uint64_t batch = 1ull << 24;
   int serial = 0;
   uint32_t pseed = 0x9E3779B9u;
@@ -182,7 +186,7 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
   // C4': default p_max = nb — eq. 3 then visits every region, so an insert fails only when
   // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
-  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax};
+  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags};
   int grid = 1, block = 32;
   if (!t->serial) {
     block = wd::kBlock;
@@ -201,7 +205,7 @@ wd_status_t launch_lane_k(wd_table* t, Shard& s, const In& in, const Out& out, u
                           cudaStream_t st) {
   auto kern = wd::probe_lane_kernel<G, K, INSERT, In, Out>;
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
-  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax};
+  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags};
   int grid = 1, block = 32;
   if (!t->serial) {
     block = wd::kBlock;
@@ -1154,6 +1158,10 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       t->kif = int(v);
       return WD_OK;
     case WD_OPT_PART_SEED: t->pseed = uint32_t(v); return WD_OK;
+    case WD_OPT_KERNEL_FLAGS:
+      if (v < 0 || v > 3) return fail(WD_ERR_INVALID_ARG, "kernel flags %lld", (long long)v);
+      t->kflags = uint32_t(v);
+      return WD_OK;
     case WD_OPT_PROBE_MODE:
       if (v < 0 || v > 2) return fail(WD_ERR_INVALID_ARG, "probe mode %lld", (long long)v);
       t->probe_mode = int(v);
@@ -1176,6 +1184,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_KEYS_IN_FLIGHT: return t->kif ? t->kif : (t->G <= 4 ? 8 : 4);
     case WD_OPT_PART_SEED: return t->pseed;
     case WD_OPT_PROBE_MODE: return t->probe_mode;
+    case WD_OPT_KERNEL_FLAGS: return t->kflags;
     case WD_OPT_PART_MODE: return t->pmode;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;

@@ -88,3 +88,21 @@ def test_query_streams():
     mq0, hit0 = wdgen.mixed_queries(5000, 2000, 0.0, seed=4)
     mq1, hit1 = wdgen.mixed_queries(5000, 2000, 1.0, seed=4)
     assert not hit0.any() and hit1.all()
+
+
+def test_zipf_frequencies_match_power_law():
+    # multiplicity of rank k ~ k^-s.  Exact sampler: frequencies within 6 sigma of
+    # p_k = k^-s / H_{N,s} for a small universe; keys are distinct per rank.
+    N, n, s = 1000, 1 << 21, 1.0 + 1e-6
+    r = wdgen.zipf_ranks(n, N, seed=3)
+    assert r.min() >= 1 and r.max() <= N
+    H = sum(k ** -s for k in range(1, N + 1))
+    cnt = np.bincount(r.astype(np.int64), minlength=N + 1)[1:]
+    for k in (1, 2, 3, 5, 10, 50, 200, 1000):
+        p = k ** -s / H
+        assert abs(cnt[k - 1] - n * p) < 6 * math.sqrt(n * p * (1 - p)) + 1, k
+    keys = wdgen.zipf_keys(1 << 16, 2**32 - 1, seed=4)
+    ranks = wdgen.zipf_ranks(1 << 16, 2**32 - 1, seed=4)
+    # rank -> key is injective (pi_s), so equal keys <=> equal ranks
+    assert np.unique(keys).size == np.unique(ranks).size
+    assert not np.any(keys == np.uint32(0xFFFFFFFF))

@@ -92,3 +92,21 @@ def test_loopback_uneven_and_empty(wd):
         assert list(gf) == [1, 1, 1, 0] and list(gv[:3]) == [3, 2, 1]
         t.insert(to_dev(np.zeros(0, np.uint32)), to_dev(np.zeros(0, np.uint32)))
         assert t.sync() == 0 and t.size() == 3
+
+
+@pytest.mark.parametrize("m", [2, 8])
+def test_loopback_zipf(wd, m):
+    # partition skew of Zipf inputs: the hottest keys all land on one shard
+    n = 1 << 19
+    keys = wdgen.zipf_keys(n, 2**32 - 1, 27)
+    vals = wdgen.values(n, 28)
+    distinct = np.unique(keys).size
+    with wd.Table(capacity_for(distinct, 0.9), group_size=4, loopback_shards=m, batch=30_000) as t:
+        q = np.unique(keys)
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0
+        assert t.size() == distinct
+    mo = oracle.Map(n, dup_mode=True)
+    mo.insert(keys, vals)
+    assert np.all(gf == 1)
+    assert np.all(mo.pair_status(q, gv) >= 1)

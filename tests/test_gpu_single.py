@@ -111,8 +111,9 @@ def test_cross_group_size(wd, Gi, Gq, mi, mq):
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
 
 
-@pytest.mark.parametrize("G,mode", [(1, 1), (4, 1), (32, 1), (2, 2), (4, 2), (8, 2), (4, 0)])
-def test_duplicates_upsert(wd, G, mode):
+@pytest.mark.parametrize("G,mode,flags", [(1, 1, 3), (4, 1, 3), (32, 1, 3), (2, 2, 3), (4, 2, 3),
+                                          (8, 2, 3), (4, 0, 3), (4, 1, 0), (4, 2, 0), (1, 1, 1)])
+def test_duplicates_upsert(wd, G, mode, flags):
     # duplicate-key mode: value must be one of the values inserted for the key;
     # size = number of distinct keys; a second stream-ordered call wins.
     n = 400_000
@@ -120,6 +121,7 @@ def test_duplicates_upsert(wd, G, mode):
     vals = wdgen.values(n, 12)
     with wd.Table(capacity_for(150_000, 0.9), 1, G) as t:
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
+        t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
         t.insert(to_dev(keys), to_dev(vals))
         q = np.arange(160_000, dtype=np.uint32)
         ov, of = t.retrieve(to_dev(q))
@@ -234,3 +236,26 @@ def test_config2_full_size_sampled(wd):
     cv, cf = oracle.expected_unique(qs, n, ks, vs)
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
     assert 0.45 < gf.mean() < 0.55
+
+
+@pytest.mark.parametrize("G,mode,flags", [(1, 1, 3), (4, 1, 3), (8, 1, 3), (4, 2, 3), (2, 2, 3),
+                                          (4, 1, 0), (4, 2, 1), (4, 1, 2)])
+def test_zipf_duplicates(wd, G, mode, flags):
+    # Zipf keys (s = 1 + 1e-6): hot keys updated by many groups at once.
+    # Every returned value must be one of the values inserted for its key; size = #distinct.
+    n = 1 << 20
+    keys = wdgen.zipf_keys(n, 2**32 - 1, 17)
+    vals = wdgen.values(n, 18)
+    distinct = np.unique(keys).size
+    with wd.Table(capacity_for(distinct, 0.95), 1, G) as t:   # load = actual occupancy
+        t.set_option(wd.WD_OPT_PROBE_MODE, mode)
+        t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
+        q = np.concatenate([np.unique(keys), wdgen.unique_keys(1000, 99)])
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0
+        assert t.size() == distinct
+    m = oracle.Map(n, dup_mode=True)
+    m.insert(keys, vals)
+    ev, ef = m.retrieve(q)
+    assert np.array_equal(gf, ef)
+    assert np.all(m.pair_status(q[gf == 1], gv[gf == 1]) >= 1)

@@ -28,7 +28,7 @@ import numpy as np
 __all__ = [
     "EMPTY_KEY", "splitmix64", "stream", "perm32", "perm32_inv", "unique_keys",
     "key_index", "values", "uniform_keys", "interleaved_queries", "mixed_queries",
-    "TAG_VAL", "TAG_UNI", "TAG_MIX", "TAG_PERM",
+    "TAG_VAL", "TAG_UNI", "TAG_MIX", "TAG_PERM", "zipf_ranks", "zipf_keys", "TAG_ZIPF",
 ]
 
 EMPTY_KEY = 0xFFFFFFFF
@@ -39,6 +39,7 @@ TAG_PERM = 0x5045524D  # "PERM"
 TAG_VAL = 0x56414C55   # "VALU"
 TAG_UNI = 0x554E4946   # "UNIF"
 TAG_MIX = 0x4D495851   # "MIXQ"
+TAG_ZIPF = 0x5A495046  # "ZIPF"
 
 _U64 = np.uint64
 
@@ -158,3 +159,64 @@ def mixed_queries(n_table: int, count: int, hit_frac: float, seed: int, start: i
     n_abs = _U64(EMPTY_KEY - n_table)
     idx = np.where(hit, r % _U64(max(n_table, 1)), _U64(n_table) + r % n_abs)
     return perm32(idx.astype(np.uint32), seed), hit
+
+
+ZIPF_S = 1.0 + 1e-6     # s = 1 + 10^-6
+ZIPF_ATTEMPTS = 8
+
+
+def _zipf_consts(universe: int, expo: float):
+    h = lambda x: np.exp(-expo * np.log(x))                                   # noqa: E731
+    hi = lambda x: _zh2((1.0 - expo) * np.log(x)) * np.log(x)                  # noqa: E731
+    hinv = lambda x: np.exp(_zh1(np.maximum(x * (1.0 - expo), -1.0)) * x)      # noqa: E731
+    c1 = hi(np.float64(1.5)) - 1.0
+    cn = hi(np.float64(universe) + 0.5)
+    sq = 2.0 - hinv(hi(np.float64(2.5)) - h(np.float64(2.0)))
+    return h, hi, hinv, c1, cn, sq
+
+
+def _zh1(x):  # log1p(x)/x
+    x = np.asarray(x, np.float64)
+    small = np.abs(x) <= 1e-8
+    xs = np.where(small, 1.0, x)
+    return np.where(small, 1 - x * (0.5 - x * (1.0 / 3 - 0.25 * x)), np.log1p(xs) / xs)
+
+
+def _zh2(x):  # expm1(x)/x
+    x = np.asarray(x, np.float64)
+    small = np.abs(x) <= 1e-8
+    xs = np.where(small, 1.0, x)
+    return np.where(small, 1 + x * 0.5 * (1 + x * (1.0 / 3) * (1 + 0.25 * x)), np.expm1(xs) / xs)
+
+
+def zipf_ranks(n: int, universe: int, seed: int, start: int = 0, expo: float = ZIPF_S):
+    """Zipf ranks k in [1, universe] with P(k) proportional to k^-s ("the
+    multiplicity of a key with rank k is smaller than the one of the most common key by a
+    factor of k^-s"; s = 1 + 1e-6).  Exact sampler: rejection-inversion (Hormann &
+    Derflinger 1996).  Sample i uses the uniforms hi53(stream(seed, ZIPF, 8 i + j)) for
+    attempts j < 8; a sample still rejected after 8 attempts (probability < 1e-9) keeps its
+    last candidate.  Implemented identically in wdgen.cu (float64)."""
+    h, hi, hinv, c1, cn, sq = _zipf_consts(universe, expo)
+    idx = np.arange(start, start + n, dtype=_U64)
+    k_out = np.zeros(n, np.uint64)
+    todo = np.ones(n, bool)
+    for j in range(ZIPF_ATTEMPTS):
+        z = stream(seed, TAG_ZIPF, idx * _U64(ZIPF_ATTEMPTS) + _U64(j))
+        uu = (z >> _U64(11)).astype(np.float64) * (1.0 / 9007199254740992.0)
+        u = cn + uu * (c1 - cn)
+        x = hinv(u)
+        k = np.floor(x + 0.5)
+        k = np.clip(k, 1, universe)
+        acc = (k - x <= sq) | (u >= hi(k + 0.5) - h(k))
+        take = todo & (acc | (j == ZIPF_ATTEMPTS - 1))
+        k_out[take] = k[take].astype(np.uint64)
+        todo &= ~take
+        if not todo.any():
+            break
+    return k_out
+
+
+def zipf_keys(n: int, universe: int, seed: int, start: int = 0):
+    """Zipf-distributed keys: rank r -> key pi_s(r - 1) (distinct ranks, distinct keys)."""
+    r = zipf_ranks(n, universe, seed, start)
+    return perm32((r - _U64(1)).astype(np.uint32), seed)

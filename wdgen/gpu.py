@@ -19,6 +19,7 @@ def lib():
         L.wdgen_uniform_keys.argtypes = [p, u64, u64, u64, p]
         L.wdgen_interleaved_queries.argtypes = [p, u64, u64, u64, u64, p]
         L.wdgen_mixed_queries.argtypes = [p, p, u64, u64, u64, C.c_double, u64, p]
+        L.wdgen_zipf_keys.argtypes = [p, u64, u64, u64, u64, p]
         _lib = L
     return _lib
 
@@ -69,4 +70,10 @@ def mixed_queries(n_table, count, hit_frac, seed, start=0, out=None, hits=None):
     hp = hits.data_ptr() if hits is not None else None
     _chk(lib().wdgen_mixed_queries(out.data_ptr(), hp, n_table, start, count, float(hit_frac),
                                    seed, _s()))
+    return out
+
+
+def zipf_keys(n, universe, seed, start=0, out=None):
+    out = _new(n) if out is None else out
+    _chk(lib().wdgen_zipf_keys(out.data_ptr(), start, n, universe, seed, _s()))
     return out

@@ -9,7 +9,7 @@
 namespace {
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr uint64_t TAG_PERM = 0x5045524D, TAG_VAL = 0x56414C55, TAG_UNI = 0x554E4946,
-                   TAG_MIX = 0x4D495851;
+                   TAG_MIX = 0x4D495851, TAG_ZIPF = 0x5A495046;
 
 __host__ __device__ inline uint64_t splitmix64(uint64_t z) {
   z += 0x9E3779B97F4A7C15ull;
@@ -80,6 +80,46 @@ __global__ void k_mixed(uint32_t* out, uint8_t* hit_out, uint64_t n_table, uint6
     if (hit_out) hit_out[i] = hit;
   }
 }
+// exact Zipf by rejection-inversion — the same computation as wdgen.zipf_ranks
+struct ZipfC { double expo, c1, cn, sq, universe; };
+__host__ __device__ inline double zh1(double x) {
+  return fabs(x) > 1e-8 ? log1p(x) / x : 1 - x * (0.5 - x * (1.0 / 3 - 0.25 * x));
+}
+__host__ __device__ inline double zh2(double x) {
+  return fabs(x) > 1e-8 ? expm1(x) / x : 1 + x * 0.5 * (1 + x * (1.0 / 3) * (1 + 0.25 * x));
+}
+__host__ __device__ inline double zh(double x, double e) { return exp(-e * log(x)); }
+__host__ __device__ inline double zhi(double x, double e) { return zh2((1.0 - e) * log(x)) * log(x); }
+__host__ __device__ inline double zhinv(double x, double e) {
+  double t = x * (1.0 - e);
+  if (t < -1.0) t = -1.0;
+  return exp(zh1(t) * x);
+}
+ZipfC zipf_consts(uint64_t universe, double e) {
+  ZipfC c;
+  c.expo = e;
+  c.universe = double(universe);
+  c.c1 = zhi(1.5, e) - 1.0;
+  c.cn = zhi(double(universe) + 0.5, e);
+  c.sq = 2.0 - zhinv(zhi(2.5, e) - zh(2.0, e), e);
+  return c;
+}
+__global__ void k_zipf(uint32_t* out, uint64_t start, uint64_t n, uint64_t sk, ZipfC c, RK rk) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x) {
+    double k = 1.0;
+    for (int j = 0; j < 8; ++j) {
+      const uint64_t z = splitmix64((start + i) * 8 + j + sk);
+      const double uu = double(z >> 11) * (1.0 / 9007199254740992.0);
+      const double u = c.cn + uu * (c.c1 - c.cn);
+      const double x = zhinv(u, c.expo);
+      k = floor(x + 0.5);
+      if (k < 1.0) k = 1.0;
+      if (k > c.universe) k = c.universe;
+      if (k - x <= c.sq || u >= zhi(k + 0.5, c.expo) - zh(k, c.expo)) break;
+    }
+    out[i] = perm32(uint32_t(uint64_t(k) - 1), rk);
+  }
+}
 int grid_for(uint64_t n) {
   uint64_t g = (n + 255) / 256;
   return int(g < 148 * 16 ? (g ? g : 1) : 148 * 16);
@@ -102,6 +142,12 @@ int wdgen_uniform_keys(uint32_t* out, uint64_t start, uint64_t n, uint64_t seed,
 int wdgen_interleaved_queries(uint32_t* out, uint64_t n_present, uint64_t start, uint64_t count,
                               uint64_t seed, cudaStream_t st) {
   if (count) k_interleaved<<<grid_for(count), 256, 0, st>>>(out, n_present, start, count, round_keys(seed));
+  return int(cudaGetLastError());
+}
+int wdgen_zipf_keys(uint32_t* out, uint64_t start, uint64_t n, uint64_t universe, uint64_t seed,
+                    cudaStream_t st) {
+  if (n) k_zipf<<<grid_for(n), 256, 0, st>>>(out, start, n, stream_key(seed, TAG_ZIPF),
+                                             zipf_consts(universe, 1.0 + 1e-6), round_keys(seed));
   return int(cudaGetLastError());
 }
 int wdgen_mixed_queries(uint32_t* out, uint8_t* hit_out, uint64_t n_table, uint64_t start, uint64_t count,
