@@ -139,7 +139,7 @@ typedef enum {
     WD_OPT_BATCH = 2,        /* items per shard per pipeline batch (2^24) */
     WD_OPT_SERIAL = 3,       /* 1: one probing group, one key at a time (deterministic
                                 layout, test hook for the Fig. 3 replay) */
-    WD_OPT_KEYS_IN_FLIGHT = 4, /* 0 = default; else keys per group in flight (4 or 8) */
+    WD_OPT_KEYS_IN_FLIGHT = 4, /* 0 = default; else keys per group in flight (1,2,4,8) */
     WD_OPT_PART_SEED = 5,    /* seed of the partition function p(k) (C15) */
     WD_OPT_PART_MODE = 6,    /* 0: p(k) = fmix32(k+seed)*m >> 32; 1: k mod m (Fig. 4) */
     WD_OPT_PROBE_MODE = 7,   /* 0 (default): auto — lane-window when the shard fits in half
@@ -150,6 +150,10 @@ typedef enum {
     WD_OPT_KERNEL_FLAGS = 8, /* bit 0: probe loads may hit L1 (safe: keys never change once
                                 written; a lost CAS reloads from L2); bit 1: value updates
                                 of existing keys as atomic exchange.  Default 3. */
+    WD_OPT_SLOTS_PER_LANE = 9, /* V: each lane of a window loads V consecutive slots with one
+                                vector load, so a window is read by |g|/V lanes (1: the
+                                paper's cooperative group; |g|: one lane).  0 = from
+                                WD_OPT_PROBE_MODE.  V in {1,2,4,8}, V <= |g|. */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -119,6 +119,7 @@ struct wd_table {
   int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit
   int kif = 0;        // keys in flight per group (0 = default)
   int probe_mode = 0; // 0: auto, 1: cooperative groups (Fig. 3), 2: lane-window (|g| <= 8)
+  int spl = 0;        // slots per lane V (WD_OPT_SLOTS_PER_LANE; 0 = from probe mode)
   // wd::kF_* kernel variants (WD_OPT_KERNEL_FLAGS).  Default both: atom.exch value updates
   // take hot (Zipf) keys from 0.5 to 6-8 G inserts/s (tools/flags_bench.py), L1-allowed
   // probe loads add ~15 % there; neither changes the unique-key rates.
@@ -179,10 +180,10 @@ int blocks_per_sm(K kern) {
 }
 
 // ------------------------------------------------------------------ probe dispatch
-template <int G, int K, bool INSERT, class In, class Out>
+template <int G, int V, int K, bool INSERT, class In, class Out>
 wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
-  auto kern = wd::probe_kernel<G, K, INSERT, In, Out>;
+  auto kern = wd::probe_kernel<G, V, K, INSERT, In, Out>;
   // C4': default p_max = nb — eq. 3 then visits every region, so an insert fails only when
   // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
@@ -190,7 +191,7 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
   int grid = 1, block = 32;
   if (!t->serial) {
     block = wd::kBlock;
-    const uint64_t keys_per_block = uint64_t(wd::kBlock / 32) * K * (32 / G);
+    const uint64_t keys_per_block = uint64_t(wd::kBlock / 32) * K * (32 / (G / V));
     const uint64_t need = std::max<uint64_t>(1, (n_hint + keys_per_block - 1) / keys_per_block);
     grid = static_cast<int>(std::min<uint64_t>(need, uint64_t(t->sm_count) * blocks_per_sm(kern)));
   }
@@ -200,62 +201,67 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
   return WD_OK;
 }
 
-template <int G, int K, bool INSERT, class In, class Out>
-wd_status_t launch_lane_k(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
-                          cudaStream_t st) {
-  auto kern = wd::probe_lane_kernel<G, K, INSERT, In, Out>;
-  const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
-  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags};
-  int grid = 1, block = 32;
-  if (!t->serial) {
-    block = wd::kBlock;
-    const uint64_t keys_per_block = uint64_t(wd::kBlock) * K;
-    const uint64_t need = std::max<uint64_t>(1, (n_hint + keys_per_block - 1) / keys_per_block);
-    grid = static_cast<int>(std::min<uint64_t>(need, uint64_t(t->sm_count) * blocks_per_sm(kern)));
+// instantiated (|g|, V, K) combinations: V = slots per lane (1: the paper's cooperative
+// group of |g| lanes; |g|: one lane per window), K = keys in flight per group
+template <int G, int V, bool INSERT, class In, class Out>
+wd_status_t launch_gv(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
+                      cudaStream_t st, int k) {
+  if constexpr (V == 1) {
+    if (k == 2) return launch_probe_k<G, 1, 2, INSERT>(t, s, in, out, n_hint, st);
+    if (k == 4) return launch_probe_k<G, 1, 4, INSERT>(t, s, in, out, n_hint, st);
+    return launch_probe_k<G, 1, 8, INSERT>(t, s, in, out, n_hint, st);
+  } else if constexpr (V == 2) {
+    if (k <= 4) return launch_probe_k<G, 2, 4, INSERT>(t, s, in, out, n_hint, st);
+    return launch_probe_k<G, 2, 8, INSERT>(t, s, in, out, n_hint, st);
+  } else if constexpr (V == 4) {
+    if (k <= 2) return launch_probe_k<G, 4, 2, INSERT>(t, s, in, out, n_hint, st);
+    return launch_probe_k<G, 4, 4, INSERT>(t, s, in, out, n_hint, st);
+  } else {
+    return launch_probe_k<G, 8, 2, INSERT>(t, s, in, out, n_hint, st);
   }
-  kern<<<grid, block, 0, st>>>(tv, in, out, s.counters, t->serial);
-  CK(cudaGetLastError());
-  t->launches++;
-  return WD_OK;
 }
 
-// lane-window keys in flight per lane: window registers grow with |g| (8|g| bytes each)
-int lane_k(int G, int kif) {
-  if (kif == 1 || kif == 2 || kif == 4 || kif == 8) {
-    if (G >= 8 && kif == 8) return 4;
-    return kif;
+// Slots per lane V (window read by |g|/V lanes) and keys in flight K for this call.
+// Explicit WD_OPT_SLOTS_PER_LANE / WD_OPT_KEYS_IN_FLIGHT win; probe mode 1 forces the
+// paper's cooperative group (V = 1), mode 2 one lane per window (V = |g| <= 8).  Auto,
+// from measurements on B200 (tools/kbench.py split, profiles/r01_split.txt):
+//  * shard in half the L2 (<= 64 MB): one lane per window, K = 2 for 32/64-byte windows —
+//    instruction-lean (e.g. |g| = 8: 18 G inserts/s, 32 G queries/s at 2^22 keys);
+//  * from HBM: two lanes per window (V = min(|g|/2, 4)), K = 4 — a warp step then waits for
+//    the slowest of 16 loads, not 32, with half the instructions of V = 1
+//    (|g| = 8, alpha 0.95, 2^28: 12.9 G inserts/s, 23.4 G queries/s vs 9.8 / 12.1 at V = 1).
+int choose_v(const wd_table* t, const Shard& s, int G) {
+  int v = t->spl;
+  if (v == 0) {
+    const bool small = s.cap * sizeof(unsigned long long) <= (64ull << 20);
+    if (t->probe_mode == 1) v = 1;
+    else if (t->probe_mode == 2 || small) v = G;
+    else v = G >= 2 ? std::max(1, std::min(G / 2, 4)) : 1;
+    if (G == 2 && t->probe_mode == 0) v = 2;
   }
-  if (G >= 8) return 2;
-  if (G == 4) return 4;
-  return 8;
+  v = std::min(v, std::min(G, 8));
+  return v;
+}
+int choose_k(const wd_table* t, const Shard& s, int G, int V) {
+  if (t->kif) return t->kif;
+  const bool small = s.cap * sizeof(unsigned long long) <= (64ull << 20);
+  if (V == 1) return G <= 4 ? 8 : 4;
+  if (V == 2) return small ? 4 : (G <= 2 ? 8 : 4);
+  if (V == 4) return small ? 2 : 4;
+  return 2;
 }
 
 template <int G, bool INSERT, class In, class Out>
 wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
-  if constexpr (G <= 8) {
-    // auto: the lane-window kernel issues 32/|g| x fewer instructions per window and wins
-    // when the table is L2-resident (measured 2-4x); from HBM the cooperative-group kernel
-    // keeps the tail of each warp step shorter (max over 32/|g| loads, not 32) and wins.
-    const bool lane = t->probe_mode == 2 ||
-                      (t->probe_mode == 0 && s.cap * sizeof(unsigned long long) <= (64ull << 20));
-    if (lane) {
-      const int k = lane_k(G, t->kif);
-      if (k == 1) return launch_lane_k<G, 1, INSERT>(t, s, in, out, n_hint, st);
-      if (k == 2) return launch_lane_k<G, 2, INSERT>(t, s, in, out, n_hint, st);
-      if constexpr (G == 8) {
-        return launch_lane_k<G, 4, INSERT>(t, s, in, out, n_hint, st);
-      } else {
-        if (k == 8) return launch_lane_k<G, 8, INSERT>(t, s, in, out, n_hint, st);
-        return launch_lane_k<G, 4, INSERT>(t, s, in, out, n_hint, st);
-      }
-    }
-  }
-  int k = t->kif;
-  if (k == 0) k = G <= 4 ? 8 : 4;   // measured on B200 (tools/gpu_run3.sh sweep)
-  if (k == 2) return launch_probe_k<G, 2, INSERT>(t, s, in, out, n_hint, st);
-  if (k == 4) return launch_probe_k<G, 4, INSERT>(t, s, in, out, n_hint, st);
-  return launch_probe_k<G, 8, INSERT>(t, s, in, out, n_hint, st);
+  const int v = choose_v(t, s, G), k = choose_k(t, s, G, v);
+  if constexpr (G >= 8)
+    if (v == 8) return launch_gv<G, 8, INSERT>(t, s, in, out, n_hint, st, k);
+  if constexpr (G >= 4)
+    if (v == 4) return launch_gv<G, 4, INSERT>(t, s, in, out, n_hint, st, k);
+  if constexpr (G >= 2)
+    if (v == 2) return launch_gv<G, 2, INSERT>(t, s, in, out, n_hint, st, k);
+  return launch_gv<G, 1, INSERT>(t, s, in, out, n_hint, st, k);
 }
 
 template <bool INSERT, class In, class Out>
@@ -1158,6 +1164,11 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       t->kif = int(v);
       return WD_OK;
     case WD_OPT_PART_SEED: t->pseed = uint32_t(v); return WD_OK;
+    case WD_OPT_SLOTS_PER_LANE:
+      if (v != 0 && v != 1 && v != 2 && v != 4 && v != 8)
+        return fail(WD_ERR_INVALID_ARG, "slots per lane %lld", (long long)v);
+      t->spl = int(v);
+      return WD_OK;
     case WD_OPT_KERNEL_FLAGS:
       if (v < 0 || v > 3) return fail(WD_ERR_INVALID_ARG, "kernel flags %lld", (long long)v);
       t->kflags = uint32_t(v);
@@ -1181,10 +1192,11 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_P_MAX: return t->pmax;
     case WD_OPT_BATCH: return int64_t(t->batch);
     case WD_OPT_SERIAL: return t->serial;
-    case WD_OPT_KEYS_IN_FLIGHT: return t->kif ? t->kif : (t->G <= 4 ? 8 : 4);
+    case WD_OPT_KEYS_IN_FLIGHT: return t->kif;
     case WD_OPT_PART_SEED: return t->pseed;
     case WD_OPT_PROBE_MODE: return t->probe_mode;
     case WD_OPT_KERNEL_FLAGS: return t->kflags;
+    case WD_OPT_SLOTS_PER_LANE: return t->spl;
     case WD_OPT_PART_MODE: return t->pmode;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;

@@ -259,3 +259,49 @@ def test_zipf_duplicates(wd, G, mode, flags):
     ev, ef = m.retrieve(q)
     assert np.array_equal(gf, ef)
     assert np.all(m.pair_status(q[gf == 1], gv[gf == 1]) >= 1)
+
+
+SPLITS = [(2, 2), (4, 2), (8, 2), (8, 4), (16, 4), (32, 8), (16, 2), (32, 4)]   # (|g|, V)
+
+
+@pytest.mark.parametrize("G,V", SPLITS)
+def test_window_split_serial_layout(wd, G, V):
+    # a window read by |g|/V lanes of V slots each: same probing, same sequential layout
+    n = 2500
+    c = oracle.physical_capacity(2700)
+    keys = np.concatenate([wdgen.unique_keys(n, 31), wdgen.unique_keys(100, 31)])
+    vals = wdgen.values(n + 100, 32)
+    r = oracle.Replay(c, G)
+    r.insert(keys, vals)
+    with wd.Table(2700, 1, G) as t:
+        t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
+        t.set_option(wd.WD_OPT_SERIAL, 1)
+        t.insert(to_dev(keys), to_dev(vals))
+        assert t.sync() == 0
+        assert np.array_equal(t.dump(), r.table)
+
+
+@pytest.mark.parametrize("G,V", SPLITS)
+def test_window_split_parity(wd, G, V):
+    n = 400_003
+    keys, vals = wdgen.unique_keys(n, 33), wdgen.values(n, 34)
+    q = wdgen.interleaved_queries(n, 33)
+    with wd.Table(capacity_for(n, 0.97), 1, G) as t:
+        t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0 and t.size() == n
+    cv, cf = oracle.expected_unique(q, n, 33, 34)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+    # duplicates through the same split
+    dk = wdgen.uniform_keys(200_000, 35) % np.uint32(60_000)
+    dv = wdgen.values(200_000, 36)
+    with wd.Table(capacity_for(60_000, 0.9), 1, G) as t:
+        t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
+        qq = np.arange(61_000, dtype=np.uint32)
+        gv, gf = gpu_roundtrip(t, dk, dv, qq)
+        m = oracle.Map(200_000, dup_mode=True)
+        m.insert(dk, dv)
+        assert t.size() == m.size()
+    ev, ef = m.retrieve(qq)
+    assert np.array_equal(gf, ef)
+    assert np.all(m.pair_status(qq[gf == 1], gv[gf == 1]) >= 1)

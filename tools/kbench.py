@@ -12,7 +12,7 @@ import paper_conf_ipps_junger0s18_b200 as wd  # noqa: E402
 import wdgen.gpu as gg  # noqa: E402
 
 
-def rate(n, G, mode, alpha=0.95, kif=0, reps=5):
+def rate(n, G, mode, alpha=0.95, kif=0, reps=5, spl=0):
     keys, vals = gg.unique_keys(n, 1), gg.values(n, 2)
     vo = torch.empty(n, dtype=torch.int32, device="cuda")
     fo = torch.empty(n, dtype=torch.uint8, device="cuda")
@@ -20,6 +20,8 @@ def rate(n, G, mode, alpha=0.95, kif=0, reps=5):
     t.set_option(wd.WD_OPT_PROBE_MODE, mode)
     if kif:
         t.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, kif)
+    if spl:
+        t.set_option(wd.WD_OPT_SLOTS_PER_LANE, spl)
     s = torch.cuda.current_stream()
     ti, tq = [], []
     for r in range(reps + 1):
@@ -34,7 +36,7 @@ def rate(n, G, mode, alpha=0.95, kif=0, reps=5):
     return n / (sum(ti) / len(ti)) / 1e6, n / (sum(tq) / len(tq)) / 1e6
 
 
-if __name__ == "__main__" and (len(sys.argv) < 2 or sys.argv[1] != "noout"):
+if __name__ == "__main__" and (len(sys.argv) < 2 or sys.argv[1] not in ("noout", "split")):
     if len(sys.argv) > 1 and sys.argv[1] == "k":
         lg = int(sys.argv[2]) if len(sys.argv) > 2 else 28
         for G, m, ks in [(4, 1, (2, 4, 8)), (4, 2, (1, 2, 4, 8)), (8, 2, (1, 2, 4)),
@@ -77,3 +79,13 @@ if __name__ == "__main__" and len(sys.argv) > 1 and sys.argv[1] == "noout":
     for G, m, k in [(4, 1, 8), (4, 2, 4), (4, 2, 1), (8, 1, 4), (8, 2, 2), (1, 2, 8)]:
         print(f"G={G} mode={m} K={k}: query without outputs {query_no_out(1 << 28, G, m, k):6.2f} G/s; "
               f"with: {rate(1 << 28, G, m, kif=k)[1]:6.2f} G/s", flush=True)
+
+
+if __name__ == "__main__" and len(sys.argv) > 1 and sys.argv[1] == "split":
+    lg = int(sys.argv[2]) if len(sys.argv) > 2 else 28
+    for G, V, ks in [(4, 1, (4, 8)), (4, 2, (4, 8)), (4, 4, (2, 4)), (8, 1, (4, 8)), (8, 2, (4, 8)),
+                     (8, 4, (2, 4)), (8, 8, (2,)), (2, 1, (4, 8)), (2, 2, (4, 8)), (16, 2, (4, 8)),
+                     (16, 4, (2, 4))]:
+        for k in ks:
+            i, q = rate(1 << lg, G, 0, kif=k, spl=V)
+            print(f"n=2^{lg} G={G} V={V} K={k}: insert {i:6.2f} G/s  query {q:6.2f} G/s", flush=True)
