@@ -1,0 +1,25 @@
+"""Small runs of every path for compute-sanitizer (memcheck / racecheck / synccheck)."""
+import os, sys
+R = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, R); sys.path.insert(0, os.path.join(R, "tests"))
+import numpy as np, torch
+import paper_conf_ipps_junger0s18_b200 as wd, wdgen, oracle
+from wdtest import gpu_roundtrip, capacity_for
+n = 20_000
+keys, vals = wdgen.unique_keys(n, 1), wdgen.values(n, 2)
+q = wdgen.interleaved_queries(n, 1)
+cv, cf = oracle.expected_unique(q, n, 1, 2)
+def check(gv, gf):
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+for G, V in [(4, 1), (8, 4), (4, 4), (1, 1), (32, 8)]:
+    with wd.Table(capacity_for(n, 0.9), 1, G) as t:
+        t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
+        check(*gpu_roundtrip(t, keys, vals, q))
+with wd.Table(capacity_for(n, 0.9), 1, 4) as t:
+    t.set_option(wd.WD_OPT_SERIAL, 1)
+    check(*gpu_roundtrip(t, keys, vals, q))
+with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=3, batch=3000) as t:
+    check(*gpu_roundtrip(t, keys, vals, q))
+with wd.Table(capacity_for(n, 0.9), 1, 8, batch=3000) as t:
+    check(*gpu_roundtrip(t, keys, vals, q, host=True))
+print("sanitize run ok")
