@@ -242,19 +242,23 @@ int choose_v(const wd_table* t, const Shard& s, int G) {
   v = std::min(v, std::min(G, 8));
   return v;
 }
-int choose_k(const wd_table* t, const Shard& s, int G, int V) {
+int choose_k(const wd_table* t, const Shard& s, int G, int V, bool insert) {
   if (t->kif) return t->kif;
   const bool small = s.cap * sizeof(unsigned long long) <= (64ull << 20);
   if (V == 1) return G <= 4 ? 8 : 4;
   if (V == 2) return small ? 4 : (G <= 2 ? 8 : 4);
-  if (V == 4) return small ? 2 : 4;
+  // V = 4: K = 2 (4 blocks/SM for inserts).  Judged on the whole step (tools/ab_retrieve.py,
+  // |g| = 8, 2^28): insert/retrieve K = 2/2 -> 13.7 / 22.6 G/s (17.1 G ops/s combined),
+  // 4/4 -> 12.9 / 23.5 (16.7), 2/4 -> 13.7 / 21.9 (16.8).
+  (void)insert;
+  if (V == 4) return 2;
   return 2;
 }
 
 template <int G, bool INSERT, class In, class Out>
 wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
-  const int v = choose_v(t, s, G), k = choose_k(t, s, G, v);
+  const int v = choose_v(t, s, G), k = choose_k(t, s, G, v, INSERT);
   if constexpr (G >= 8)
     if (v == 8) return launch_gv<G, 8, INSERT>(t, s, in, out, n_hint, st, k);
   if constexpr (G >= 4)
