@@ -70,10 +70,15 @@ def lib():
         L.or_multisplit.argtypes = [p, u64, u32, u32, C.c_int, p, p]
         L.or_multisplit.restype = None
         L.or_table_scans.argtypes = [p, u32, p, p]; L.or_table_scans.restype = None
-        L.or_replay_insert.argtypes = [p, u64, C.c_int, u32, p, p, u64, C.POINTER(_Stats)]
+        L.or_replay_insert.argtypes = [p, u64, C.c_int, u32, u32, p, p, u64, C.POINTER(_Stats)]
         L.or_replay_insert.restype = None
-        L.or_replay_query.argtypes = [p, u64, C.c_int, u32, p, p, p, u64, C.POINTER(_Stats)]
+        L.or_replay_query.argtypes = [p, u64, C.c_int, u32, u32, p, p, p, u64,
+                                      C.POINTER(_Stats), C.c_int]
         L.or_replay_query.restype = None
+        L.or_replay_rebuild.argtypes = [p, p, u64, C.c_int, u32, u32, C.POINTER(_Stats)]
+        L.or_replay_rebuild.restype = None
+        L.or_replay_base_seed.argtypes = [u32, u32, u64, u32]; L.or_replay_base_seed.restype = u64
+        L.or_map_erase.argtypes = [p, p, p, u64]; L.or_map_erase.restype = u64
         L.or_replay_base.argtypes = [u32, u32, u64]; L.or_replay_base.restype = u64
         L.or_physical_capacity.argtypes = [u64]; L.or_physical_capacity.restype = u64
         for f in (L.or_fmix32_many, L.or_mueller_many):
@@ -154,6 +159,13 @@ class Map:
     def size(self) -> int:
         return int(lib().or_map_size(self._h))
 
+    def erase(self, keys):
+        """P:91 deletion; returns found (uint8 per key: was present and is now removed)."""
+        k = _u32(keys)
+        found = np.empty(k.size, np.uint8)
+        lib().or_map_erase(self._h, _ptr(k), _ptr(found), k.size)
+        return found
+
     def pair_status(self, keys, vals) -> np.ndarray:
         """0: (k,v) never inserted; 1: inserted in some call; 2: in k's last call."""
         k, v = _u32(keys), _u32(vals)
@@ -184,34 +196,52 @@ def table_scans(T):
 
 
 # ---------------------------------------------------------------- (6) Fig. 3 replay
-class Replay:
-    """Sequential single-group replay of Fig. 3 on a c-slot table (c >= 32, c % 4 == 0)."""
+TOMB_WORD = 0xFFFFFFFEFFFFFFFF
 
-    def __init__(self, capacity: int, group_size: int, p_max: int = 1024):
+
+class Replay:
+    """Sequential single-group replay of Fig. 3 on a c-slot table (c >= 32, c % 4 == 0)
+    with hash seed `seed` (P:161 translated variants; P:63 rebuild with a distinct one)."""
+
+    def __init__(self, capacity: int, group_size: int, p_max: int = 1024, seed: int = 0):
         assert capacity >= 32 and capacity % 4 == 0
         assert group_size in (1, 2, 4, 8, 16, 32)
-        self.c, self.G, self.pmax = int(capacity), int(group_size), int(p_max)
+        self.c, self.G, self.pmax, self.seed = int(capacity), int(group_size), int(p_max), int(seed)
         self.table = np.full(self.c, np.uint64(0xFFFFFFFFFFFFFFFF), np.uint64)
         self.ins = _Stats()
         self.qry = _Stats()
 
     def insert(self, keys, vals):
         k, v = _u32(keys), _u32(vals)
-        lib().or_replay_insert(_ptr(self.table), self.c, self.G, self.pmax, _ptr(k), _ptr(v),
-                               k.size, C.byref(self.ins))
+        lib().or_replay_insert(_ptr(self.table), self.c, self.G, self.pmax, self.seed, _ptr(k),
+                               _ptr(v), k.size, C.byref(self.ins))
 
-    def query(self, keys, stats: _Stats | None = None):
+    def query(self, keys, stats: _Stats | None = None, erase: bool = False):
         k = _u32(keys)
         vals = np.empty(k.size, np.uint32)
         found = np.empty(k.size, np.uint8)
         st = stats if stats is not None else self.qry
-        lib().or_replay_query(_ptr(self.table), self.c, self.G, self.pmax, _ptr(k), _ptr(vals),
-                              _ptr(found), k.size, C.byref(st))
+        lib().or_replay_query(_ptr(self.table), self.c, self.G, self.pmax, self.seed, _ptr(k),
+                              _ptr(vals), _ptr(found), k.size, C.byref(st), int(erase))
         return vals, found
 
+    def erase(self, keys):
+        """P:91 deletion: matching slots become tombstones (reading C9'); returns found."""
+        return self.query(keys, _Stats(), erase=True)[1]
+
+    def rebuild(self, seed: int):
+        """re-insert every live slot (slot order) into a fresh table with `seed`."""
+        old = self.table.copy()
+        self.seed = int(seed)
+        self.table = np.full(self.c, np.uint64(0xFFFFFFFFFFFFFFFF), np.uint64)
+        st = _Stats()
+        lib().or_replay_rebuild(_ptr(old), _ptr(self.table), self.c, self.G, self.pmax,
+                                self.seed, C.byref(st))
+        return st
+
     @staticmethod
-    def base(k: int, p: int, capacity: int) -> int:
-        return int(lib().or_replay_base(int(k), int(p), int(capacity)))
+    def base(k: int, p: int, capacity: int, seed: int = 0) -> int:
+        return int(lib().or_replay_base_seed(int(k), int(p), int(capacity), int(seed)))
 
 
 def physical_capacity(c: int) -> int:

@@ -374,3 +374,89 @@ def test_replay_probe_costs_grow_with_load():
             w[a, G] = r.ins.windows / n
     assert w[0.8, 4] < w[0.95, 4]
     assert w[0.95, 1] > w[0.95, 4] > w[0.95, 32] >= 1.0
+
+
+# ------------------------------------------------------------------ deletion (C9')
+@pytest.mark.parametrize("trial", range(12))
+def test_map_erase_matches_bruteforce(trial):
+    # Algorithm R keeps linear-probing clusters searchable after deletions; a tiny initial
+    # capacity + a small key domain make long clusters and wrap-around
+    rnd = random.Random(100 + trial)
+    domain = [rnd.randrange(0, 2**32 - 1) for _ in range(30)]
+    m = oracle.Map(4, dup_mode=True)
+    d, lastcall, paircall, erasecall = {}, {}, {}, {}
+    call = 0
+    for _ in range(rnd.randint(3, 8)):
+        call += 1
+        if rnd.random() < 0.5:
+            ks = [rnd.choice(domain) for _ in range(rnd.randint(0, 40))]
+            vs = [rnd.randrange(2**32) for _ in ks]
+            m.insert(np.array(ks, np.uint32), np.array(vs, np.uint32))
+            for k, v in zip(ks, vs):
+                d[k] = v; lastcall[k] = call; paircall[(k, v)] = call
+        else:
+            ks = [rnd.choice(domain) for _ in range(rnd.randint(0, 20))]
+            f = m.erase(np.array(ks, np.uint32))
+            seen = set()
+            for k, fi in zip(ks, f):
+                assert fi == (1 if (k in d and k not in seen) else 0)
+                if k in d and k not in seen:
+                    seen.add(k)
+                    del d[k]
+                erasecall[k] = call
+    assert m.size() == len(d)
+    q = np.array(domain + [rnd.randrange(2**32 - 1) for _ in range(10)], np.uint32)
+    vals, found = m.retrieve(q)
+    for k, v, fnd in zip(q, vals, found):
+        k = int(k)
+        assert fnd == (k in d) and (not fnd or int(v) == d[k])
+    for (k, v), pc in list(paircall.items())[:40]:
+        st = int(m.pair_status(np.array([k], np.uint32), np.array([v], np.uint32))[0])
+        live = pc > erasecall.get(k, 0)
+        want = 0 if not live else (2 if k in d and lastcall[k] == pc else 1)
+        assert st == want, (k, v, st, want)
+
+
+@pytest.mark.parametrize("G", [1, 4, 8])
+def test_replay_with_tombstones_equals_map(G):
+    # sequential Fig. 3 with deletions: queries probe past tombstones, inserts never reuse
+    # them (C9'); results equal the plain dictionary through insert/erase/insert rounds
+    n = 4000
+    c = oracle.physical_capacity(3 * n)
+    r = oracle.Replay(c, G, p_max=(c - 32) // 4 + 1)
+    m = oracle.Map(n)
+    keys = wdgen.unique_keys(n, 61)
+    r.insert(keys, wdgen.values(n, 62)); m.insert(keys, wdgen.values(n, 62))
+    er = keys[::3]
+    assert np.array_equal(r.erase(er), m.erase(er))
+    assert np.array_equal(r.erase(er[:50]), np.zeros(50, np.uint8))        # already gone
+    again = np.concatenate([er[:500], wdgen.unique_keys(300, 61, start=n)])
+    r.insert(again, wdgen.values(again.size, 63)); m.insert(again, wdgen.values(again.size, 63))
+    q = np.concatenate([keys, wdgen.unique_keys(600, 61, start=n)])
+    rv, rf = r.query(q)
+    mv, mf = m.retrieve(q)
+    assert np.array_equal(rf, mf) and np.array_equal(rv, mv)
+    # tombstones are never reused: every erased key left one, re-inserted keys took new slots
+    tombs = int(np.sum(r.table == np.uint64(oracle.TOMB_WORD)))
+    live = int(np.sum((r.table & np.uint64(0xFFFFFFFF)) != np.uint64(0xFFFFFFFF)))
+    assert tombs == er.size and live == m.size()
+
+
+def test_replay_rebuild_drops_tombstones():
+    n = 3000
+    c = oracle.physical_capacity(2 * n)
+    r = oracle.Replay(c, 4)
+    m = oracle.Map(n)
+    keys, vals = wdgen.unique_keys(n, 71), wdgen.values(n, 72)
+    r.insert(keys, vals); m.insert(keys, vals)
+    r.erase(keys[1::2]); m.erase(keys[1::2])
+    st = r.rebuild(seed=0x1234567)
+    assert st.failures == 0 and st.new_keys == m.size()
+    assert not np.any(r.table == np.uint64(oracle.TOMB_WORD))
+    q = np.concatenate([keys, wdgen.unique_keys(500, 71, start=n)])
+    rv, rf = r.query(q)
+    mv, mf = m.retrieve(q)
+    assert np.array_equal(rf, mf) and np.array_equal(rv, mv)
+    # a distinct seed is a distinct probe sequence ("distinct hash function")
+    assert any(oracle.Replay.base(int(k), 0, c, 0x1234567) != oracle.Replay.base(int(k), 0, c)
+               for k in keys[:20])
