@@ -121,6 +121,19 @@ wd_status_t wd_insert(wd_table_t* t, const uint32_t* keys, const uint32_t* vals,
 wd_status_t wd_retrieve(wd_table_t* t, const uint32_t* keys, uint32_t* vals_out,
                         uint8_t* found_out, uint64_t n, wd_stream_t stream);
 
+/* P:91 deletion (NEXT #3; barrier-separated from inserts, i.e. not concurrent with a
+ * wd_insert on the same table): every present key in keys[0..n) is removed — its slot
+ * becomes a tombstone (reading C9': probed past by queries, not reused by inserts until
+ * wd_rebuild).  found_out[i] (may be NULL) = 1 for exactly one occurrence of each key this
+ * call removed.  Same pointer kinds and asynchrony as wd_retrieve. */
+wd_status_t wd_erase(wd_table_t* t, const uint32_t* keys, uint8_t* found_out, uint64_t n,
+                     wd_stream_t stream);
+
+/* P:63 reconstruction: re-insert every live entry into a fresh table of the same capacity
+ * with the hash seed `seed` (translated variants h(k + seed)); tombstones are dropped.
+ * Synchronizes; needs a second table's worth of device memory transiently. */
+wd_status_t wd_rebuild(wd_table_t* t, uint32_t seed, wd_stream_t stream);
+
 /* a5: number of distinct keys stored (summed over shards and ranks).  Synchronizes.
  * UINT64_MAX on error. */
 uint64_t wd_size(wd_table_t* t);
@@ -174,8 +187,9 @@ uint64_t    wd_shard_capacity(wd_table_t* t, int shard);
  * word = key | (uint64_t)value << 32, empty = all ones.  Synchronizes. */
 wd_status_t wd_dump(wd_table_t* t, int shard, uint64_t* host_out);
 /* per-shard device counters: [0] new keys, [1] failed inserts, [2] reserved keys,
- * [3] exchange errors, [4] key of the most recent failed insert.  Synchronizes. */
-wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[5]);
+ * [3] exchange errors, [4] key of the most recent failed insert, [5] keys erased.
+ * Synchronizes. */
+wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[6]);
 
 #ifdef __cplusplus
 }

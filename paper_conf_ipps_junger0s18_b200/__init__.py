@@ -39,7 +39,8 @@ EXPORTS = ["wd_create", "wd_create_loopback", "wd_create_rank", "wd_rank_handle"
            "wd_rank_connect",
            "wd_destroy", "wd_clear", "wd_insert", "wd_retrieve", "wd_size", "wd_capacity",
            "wd_sync", "wd_set_option", "wd_get_option", "wd_last_error", "wd_error_string",
-           "wd_last_error_message", "wd_shard_capacity", "wd_dump", "wd_counters"]
+           "wd_last_error_message", "wd_shard_capacity", "wd_dump", "wd_counters", "wd_erase",
+           "wd_rebuild"]
 
 
 class WarpDriveError(RuntimeError):
@@ -82,6 +83,8 @@ def _load():
         "wd_shard_capacity": ([p, i32], u64),
         "wd_dump": ([p, i32, p], i32),
         "wd_counters": ([p, i32, p], i32),
+        "wd_erase": ([p, p, p, u64, p], i32),
+        "wd_rebuild": ([p, C.c_uint32, p], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -216,6 +219,24 @@ class Table:
         _check(_lib.wd_retrieve(self._h, kp, vp, fp, n, _stream(stream)))
         return vals_out, found_out
 
+    def erase(self, keys, found_out=None, stream=None):
+        """P:91 deletion; found_out[i] = 1 for the occurrence that removed keys[i]."""
+        kp, n, kc = _addr(keys)
+        if found_out is None:
+            import torch
+            if isinstance(keys, torch.Tensor):
+                pin = keys.device.type == "cpu" and keys.is_pinned()
+                found_out = torch.empty(n, dtype=torch.uint8, device=keys.device, pin_memory=pin)
+            else:
+                found_out = np.empty(n, np.uint8)
+        fp, _, _ = _addr(found_out)
+        _check(_lib.wd_erase(self._h, kp, fp, n, _stream(stream)))
+        return found_out
+
+    def rebuild(self, seed: int, stream=None):
+        """re-insert the live entries into a fresh table with hash seed `seed`."""
+        _check(_lib.wd_rebuild(self._h, int(seed) & 0xFFFFFFFF, _stream(stream)))
+
     # -- queries of state
     def size(self) -> int:
         s = _lib.wd_size(self._h)
@@ -245,10 +266,11 @@ class Table:
         return out
 
     def counters(self, shard: int = 0) -> dict:
-        out = np.zeros(5, np.uint64)
+        out = np.zeros(6, np.uint64)
         _check(_lib.wd_counters(self._h, shard, out.ctypes.data))
         return {"new": int(out[0]), "failed": int(out[1]), "reserved": int(out[2]),
-                "exchange_errors": int(out[3]), "last_failed_key": int(out[4])}
+                "exchange_errors": int(out[3]), "last_failed_key": int(out[4]),
+                "erased": int(out[5])}
 
     @property
     def launches(self) -> int:

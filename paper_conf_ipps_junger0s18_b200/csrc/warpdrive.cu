@@ -85,6 +85,7 @@ struct Shard {
   int id = 0;        // global shard index (= owner id of p(k))
   int device = 0;
   uint64_t cap = 0, nb = 0;
+  uint32_t hseed = 0;            // hash seed of the current table (changes on rebuild)
   unsigned long long* slots = nullptr;
   unsigned long long* counters = nullptr;
   cudaStream_t s_main = nullptr, s_h2d = nullptr, s_d2h = nullptr;
@@ -187,7 +188,7 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
   // C4': default p_max = nb — eq. 3 then visits every region, so an insert fails only when
   // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
-  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags};
+  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags, s.hseed};
   int grid = 1, block = 32;
   if (!t->serial) {
     block = wd::kBlock;
@@ -615,14 +616,24 @@ wd_status_t stage_out(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int sl
 bool needs_staging(const IO& io) { return io.kin != PK_DEVICE || io.kout != PK_DEVICE; }
 
 // ------------------------------------------------------------------ single-shard path
-wd_status_t single_op(wd_table* t, bool insert, const IO& io, cudaStream_t stream) {
+enum Op { OP_INSERT = 0, OP_RETRIEVE = 1, OP_ERASE = 2 };
+
+// the probe kernel of one call on a plain (SoA) input
+wd_status_t probe_soa(wd_table* t, Shard& s, int op, const wd::InSoA& in, uint32_t* ov, uint8_t* of,
+                      uint64_t n, cudaStream_t st) {
+  if (op == OP_INSERT) return launch_probe<true>(t, s, in, wd::OutNone{}, n, st);
+  if (op == OP_ERASE) return launch_probe<false>(t, s, in, wd::OutErase<wd::OutSoA>{{nullptr, of}}, n, st);
+  return launch_probe<false>(t, s, in, wd::OutSoA{ov, of}, n, st);
+}
+
+wd_status_t single_op(wd_table* t, int op, const IO& io, cudaStream_t stream) {
+  const bool insert = op == OP_INSERT;
   Shard& s = t->local[0];
   DeviceGuard g(s.device);
   if (!needs_staging(io)) {  // device-resident: one kernel on the caller's stream
     if (io.n == 0) return WD_OK;
     const wd::InSoA in{io.keys, io.vals, io.n};
-    if (insert) return launch_probe<true>(t, s, in, wd::OutNone{}, io.n, stream);
-    return launch_probe<false>(t, s, in, wd::OutSoA{io.vout, io.fout}, io.n, stream);
+    return probe_soa(t, s, op, in, io.vout, io.fout, io.n, stream);
   }
   // out-of-core pipeline (Fig. 5): H2D(b+1) || probe(b) || D2H(b-1)
   const uint64_t B = t->batch;
@@ -637,13 +648,9 @@ wd_status_t single_op(wd_table* t, bool insert, const IO& io, cudaStream_t strea
     const uint32_t *dk, *dv;
     TRY(stage_in(s, io, off, cnt, slot, insert, &dk, &dv));
     const wd::InSoA in{dk, dv, cnt};
-    if (insert) {
-      TRY(launch_probe<true>(t, s, in, wd::OutNone{}, cnt, s.s_main));
-    } else {
-      uint32_t* ov; uint8_t* of;
-      out_ptrs(s, io, off, slot, &ov, &of);
-      TRY(launch_probe<false>(t, s, in, wd::OutSoA{ov, of}, cnt, s.s_main));
-    }
+    uint32_t* ov = nullptr; uint8_t* of = nullptr;
+    if (!insert) out_ptrs(s, io, off, slot, &ov, &of);
+    TRY(probe_soa(t, s, op, in, ov, of, cnt, s.s_main));
     TRY(stage_out(s, io, off, cnt, slot, !insert));
   }
   return join_into(t, stream, ev0);
@@ -677,7 +684,8 @@ wd_status_t agree_batches(wd_table* t, uint64_t local_nbt, uint64_t* global_nbt)
   return WD_OK;
 }
 
-wd_status_t cascade_op(wd_table* t, bool insert, std::vector<IO>& ios, cudaStream_t stream) {
+wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t stream) {
+  const bool insert = op == OP_INSERT;
   TRY(ensure_exchange(t));
   const uint64_t B = t->batch;
   const int m = t->m;
@@ -756,7 +764,10 @@ wd_status_t cascade_op(wd_table* t, bool insert, std::vector<IO>& ios, cudaStrea
         // origins consumed the results of the previous query epoch that used this slot
         if (t->res_used[slot]) TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
         const wd::InSeg<false> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
-        TRY(launch_probe<false>(t, s, in, wd::OutPacked{s.self.res[slot]}, B, s.s_probe));
+        if (op == OP_ERASE)
+          TRY(launch_probe<false>(t, s, in, wd::OutErase<wd::OutPacked>{{s.self.res[slot]}}, B, s.s_probe));
+        else
+          TRY(launch_probe<false>(t, s, in, wd::OutPacked{s.self.res[slot]}, B, s.s_probe));
       }
       TRY(launch_signal(t, s, s.s_probe, FLAG_DONE, e));
     }
@@ -828,8 +839,9 @@ wd_status_t check_ptr(wd_table* t, const void* p, PtrKind* kind) {
   return WD_OK;
 }
 
-wd_status_t do_op(wd_table* t, bool insert, const uint32_t* keys, const uint32_t* vals,
+wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* vals,
                   uint32_t* vout, uint8_t* fout, uint64_t n, cudaStream_t stream) {
+  const bool insert = op == OP_INSERT;
   if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
   if (n && !keys) return fail(WD_ERR_INVALID_ARG, "keys == NULL with n > 0");
   if (n && insert && !vals) return fail(WD_ERR_INVALID_ARG, "vals == NULL with n > 0");
@@ -853,11 +865,11 @@ wd_status_t do_op(wd_table* t, bool insert, const uint32_t* keys, const uint32_t
   }
   if (t->m == 1) {
     if (n == 0) return WD_OK;
-    return single_op(t, insert, io, stream);
+    return single_op(t, op, io, stream);
   }
   std::vector<IO> ios;
   split_io(t, io, ios);
-  return cascade_op(t, insert, ios, stream);
+  return cascade_op(t, op, ios, stream);
 }
 
 wd_table* create_common(uint64_t capacity, int mode, int m, int group_size) {
@@ -900,7 +912,7 @@ uint64_t shard_cap(uint64_t capacity, int m) {
 }
 
 wd_status_t sticky_status(wd_table* t) {
-  unsigned long long agg[wd::CNT_N] = {0, 0, 0, 0, 0};
+  unsigned long long agg[wd::CNT_N] = {};
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
     unsigned long long c[wd::CNT_N];
@@ -1106,13 +1118,53 @@ wd_status_t wd_clear(wd_table_t* t, wd_stream_t stream) {
 
 wd_status_t wd_insert(wd_table_t* t, const uint32_t* keys, const uint32_t* vals, uint64_t n,
                       wd_stream_t stream) {
-  return do_op(t, true, keys, vals, nullptr, nullptr, n, reinterpret_cast<cudaStream_t>(stream));
+  return do_op(t, OP_INSERT, keys, vals, nullptr, nullptr, n, reinterpret_cast<cudaStream_t>(stream));
 }
 
 wd_status_t wd_retrieve(wd_table_t* t, const uint32_t* keys, uint32_t* vals_out, uint8_t* found_out,
                         uint64_t n, wd_stream_t stream) {
-  return do_op(t, false, keys, nullptr, vals_out, found_out, n,
+  return do_op(t, OP_RETRIEVE, keys, nullptr, vals_out, found_out, n,
                reinterpret_cast<cudaStream_t>(stream));
+}
+
+wd_status_t wd_erase(wd_table_t* t, const uint32_t* keys, uint8_t* found_out, uint64_t n,
+                     wd_stream_t stream) {
+  return do_op(t, OP_ERASE, keys, nullptr, nullptr, found_out, n,
+               reinterpret_cast<cudaStream_t>(stream));
+}
+
+wd_status_t wd_rebuild(wd_table_t* t, uint32_t seed, wd_stream_t stream) {
+  if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    CK(cudaStreamSynchronize(st));
+    CK(cudaDeviceSynchronize());
+    // 1. gather the live slots (the contents survive, tombstones do not)
+    unsigned long long *live = nullptr, *cnt = nullptr, *fresh = nullptr;
+    CK(cudaMalloc(&live, s.cap * sizeof(unsigned long long)));
+    CK(cudaMalloc(&cnt, sizeof(unsigned long long)));
+    CK(cudaMalloc(&fresh, s.cap * sizeof(unsigned long long)));
+    CK(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long), s.s_main));
+    const int cgrid = t->serial ? 1 : t->sm_count * 8;
+    wd::compact_kernel<<<cgrid, t->serial ? 32 : wd::kBlock, 0, s.s_main>>>(s.slots, s.cap, live, cnt);
+    CK(cudaGetLastError());
+    // 2. a fresh table with the distinct hash (translated variant)
+    wd::fill_kernel<<<t->sm_count * 4, wd::kBlock, 0, s.s_main>>>(fresh, s.cap, s.counters, wd::CNT_N);
+    CK(cudaGetLastError());
+    t->launches += 2;
+    unsigned long long* old = s.slots;
+    s.slots = fresh;
+    s.hseed = seed;
+    // 3. re-insert (Fig. 3) from the gathered pairs
+    const wd::InSeg<true> in{live, cnt, s.cap, 1};
+    TRY(launch_probe<true>(t, s, in, wd::OutNone{}, s.cap, s.s_main));
+    CK(cudaStreamSynchronize(s.s_main));
+    cudaFree(old);
+    cudaFree(live);
+    cudaFree(cnt);
+  }
+  return WD_OK;
 }
 
 wd_status_t wd_sync(wd_table_t* t) {
@@ -1125,13 +1177,13 @@ uint64_t wd_size(wd_table_t* t) {
   unsigned long long total = 0;
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
-    unsigned long long c = 0;
+    unsigned long long c[wd::CNT_N];
     if (cudaDeviceSynchronize() != cudaSuccess ||
-        cudaMemcpy(&c, s.counters + wd::CNT_NEW, 8, cudaMemcpyDeviceToHost) != cudaSuccess) {
+        cudaMemcpy(c, s.counters, sizeof c, cudaMemcpyDeviceToHost) != cudaSuccess) {
       fail(WD_ERR_CUDA, "wd_size: %s", cudaGetErrorString(cudaGetLastError()));
       return UINT64_MAX;
     }
-    total += c;
+    total += c[wd::CNT_NEW] - c[wd::CNT_ERASED];
   }
   if (t->mode == MODE_RANK) {
     uint64_t v = total;
@@ -1245,7 +1297,7 @@ wd_status_t wd_dump(wd_table_t* t, int shard, uint64_t* host_out) {
   return WD_OK;
 }
 
-wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[5]) {
+wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[6]) {
   if (!t || shard < 0 || shard >= int(t->local.size()) || !out)
     return fail(WD_ERR_INVALID_ARG, "wd_counters arguments");
   Shard& s = t->local[shard];
