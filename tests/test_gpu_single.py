@@ -305,3 +305,29 @@ def test_window_split_parity(wd, G, V):
     ev, ef = m.retrieve(qq)
     assert np.array_equal(gf, ef)
     assert np.all(m.pair_status(qq[gf == 1], gv[gf == 1]) >= 1)
+
+
+def test_config3_single_gpu_full_size(wd):
+    # BASELINE config 3 at m = 1: every non-sentinel 4-byte key (n = 2^32 - 1, C14) into a
+    # 4.52e9-slot table (36 GB, 64-bit slot indices) at alpha 0.95; inputs generated on the
+    # device; a 2^21 random sample of queries checked against the closed form.
+    import torch
+    import wdgen.gpu as gg
+    free, _ = torch.cuda.mem_get_info()
+    if free < 100e9:
+        pytest.skip("needs ~90 GB of device memory")
+    n = (1 << 32) - 1
+    keys, vals = gg.unique_keys(n, 111), gg.values(n, 112)
+    with wd.Table(capacity_for(n, 0.95), 1, 8) as t:
+        t.insert(keys, vals)
+        del vals
+        torch.cuda.synchronize()
+        assert t.sync() == 0 and t.size() == n
+        idx = torch.randint(0, n, (1 << 21,), device="cuda", dtype=torch.int64)
+        q = torch.cat([keys[idx], gg.unique_keys(1 << 10, 999)])   # + keys of another seed
+        ov, of = t.retrieve(q)
+        torch.cuda.synchronize()
+        gv, gf = from_dev(ov), of.cpu().numpy()
+        qs = from_dev(q)
+    cv, cf = oracle.expected_unique(qs, n, 111, 112)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
