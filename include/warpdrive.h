@@ -71,7 +71,8 @@ typedef enum {
  * peer access over NVLink; host input is split into n_gpus contiguous chunks.
  * capacity: total slots c (alpha = n / c).  Each shard gets ceil(c / m) slots,
  * rounded up to a multiple of 4 and to at least 32 (the 32-slot region, Fig. 3 Line 6).
- * group_size: |g| in {1,2,4,8,16,32}.  Returns NULL on error (see wd_last_error). */
+ * group_size: |g| in {1,2,4,8,16,32}, or 0 = dynamic by load (see
+ * WD_OPT_GROUP_SIZE).  Returns NULL on error (see wd_last_error). */
 wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size);
 
 /* Test backend: m virtual shards on the CURRENT device, running the full multi-GPU
@@ -146,7 +147,9 @@ wd_status_t wd_sync(wd_table_t* t);
 
 /* ------------------------------------------------------------------ options -------- */
 typedef enum {
-    WD_OPT_GROUP_SIZE = 0,   /* |g|; the probe sequence does not depend on it */
+    WD_OPT_GROUP_SIZE = 0,   /* |g|; the probe sequence does not depend on it.
+                                0 = dynamic by load: 8, or 16 above a projected
+                                load of 0.97 (measured on B200) */
     WD_OPT_P_MAX = 1,        /* outer probing bound p_max (Fig. 3 Line 4); 0 (default) = the
                                 number of regions nb, i.e. fail only when the table is full (C4') */
     WD_OPT_BATCH = 2,        /* items per shard per pipeline batch (2^24) */
@@ -170,7 +173,8 @@ typedef enum {
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */
-    WD_OPT_LAUNCHES = 103    /* read-only: kernels launched by the library so far */
+    WD_OPT_LAUNCHES = 103,   /* read-only: kernels launched by the library so far */
+    WD_OPT_GROUP_SIZE_USED = 104 /* read-only: |g| used by the last call */
 } wd_option_t;
 
 wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t value);

@@ -116,7 +116,9 @@ struct wd_table {
   int mode = MODE_SINGLE;
   int m = 1;          // number of shards (= GPUs, or virtual shards in loopback)
   int rank = 0;       // rank mode: this process's shard id
-  int G = 4;
+  int G = 4;          // |g|, or 0 = dynamic by load
+  int G_used = 4;     // |g| of the current / last call
+  uint64_t est_size = 0;   // host-side upper estimate of the stored keys (no sync needed)
   int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit
   int kif = 0;        // keys in flight per group (0 = default)
   int probe_mode = 0; // 0: auto, 1: cooperative groups (Fig. 3), 2: lane-window (|g| <= 8)
@@ -272,7 +274,7 @@ wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, 
 template <bool INSERT, class In, class Out>
 wd_status_t launch_probe(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                          cudaStream_t st) {
-  switch (t->G) {
+  switch (t->G_used) {
     case 1: return launch_probe_g<1, INSERT>(t, s, in, out, n_hint, st);
     case 2: return launch_probe_g<2, INSERT>(t, s, in, out, n_hint, st);
     case 4: return launch_probe_g<4, INSERT>(t, s, in, out, n_hint, st);
@@ -280,7 +282,7 @@ wd_status_t launch_probe(wd_table* t, Shard& s, const In& in, const Out& out, ui
     case 16: return launch_probe_g<16, INSERT>(t, s, in, out, n_hint, st);
     case 32: return launch_probe_g<32, INSERT>(t, s, in, out, n_hint, st);
   }
-  return fail(WD_ERR_INVALID_ARG, "group size %d not in {1,2,4,8,16,32}", t->G);
+  return fail(WD_ERR_INVALID_ARG, "group size %d not in {1,2,4,8,16,32}", t->G_used);
 }
 
 // ------------------------------------------------------------------ shard lifetime
@@ -863,6 +865,17 @@ wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* val
     io.kout = insert ? PK_DEVICE : (vout ? k2 : k3);
     if (!insert && !vout && !fout) io.kout = PK_DEVICE;
   }
+  // P:245 future work, built: "a heuristic which dynamically scales the group size |g|
+  // with the current load factor".  P:89 makes switching |g| between calls safe (same probe
+  // sequence).  Measured on B200 (profiles/r01_sweep.jsonl, 2^28 keys): |g| = 8 is fastest
+  // up to alpha ~0.95, |g| = 16 at 0.99.  The load used is the projected one after this call,
+  // from a host-side upper estimate of the size (no synchronisation).
+  if (t->G == 0) {
+    const double cap = double(wd_capacity(t));
+    const double est = double(t->est_size) + (op == OP_INSERT ? double(n) : 0.0);
+    t->G_used = (est / cap > 0.97) ? 16 : 8;
+  }
+  if (op == OP_INSERT) t->est_size = std::min<uint64_t>(t->est_size + n, wd_capacity(t));
   if (t->m == 1) {
     if (n == 0) return WD_OK;
     return single_op(t, op, io, stream);
@@ -874,9 +887,9 @@ wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* val
 
 wd_table* create_common(uint64_t capacity, int mode, int m, int group_size) {
   if (capacity < 1) { fail(WD_ERR_INVALID_ARG, "capacity must be >= 1"); return nullptr; }
-  if (group_size != 1 && group_size != 2 && group_size != 4 && group_size != 8 &&
-      group_size != 16 && group_size != 32) {
-    fail(WD_ERR_INVALID_ARG, "group_size %d not in {1,2,4,8,16,32}", group_size);
+  if (group_size != 0 && group_size != 1 && group_size != 2 && group_size != 4 &&
+      group_size != 8 && group_size != 16 && group_size != 32) {
+    fail(WD_ERR_INVALID_ARG, "group_size %d not in {0 (auto),1,2,4,8,16,32}", group_size);
     return nullptr;
   }
   if (m < 1 || m > wd::kMaxShards) {
@@ -887,6 +900,7 @@ wd_table* create_common(uint64_t capacity, int mode, int m, int group_size) {
   t->mode = mode;
   t->m = m;
   t->G = group_size;
+  t->G_used = group_size ? group_size : 8;
   return t;
 }
 
@@ -1095,6 +1109,7 @@ void wd_destroy(wd_table_t* t) {
 
 wd_status_t wd_clear(wd_table_t* t, wd_stream_t stream) {
   if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  t->est_size = 0;
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   if (t->mode == MODE_SINGLE) {
     Shard& s = t->local[0];
@@ -1190,6 +1205,7 @@ uint64_t wd_size(wd_table_t* t) {
     if (host_allreduce(t, &v, WD_REDUCE_SUM) != WD_OK) return UINT64_MAX;
     total = v;
   }
+  t->est_size = total;
   return total;
 }
 
@@ -1202,9 +1218,10 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
   if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
   switch (opt) {
     case WD_OPT_GROUP_SIZE:
-      if (v != 1 && v != 2 && v != 4 && v != 8 && v != 16 && v != 32)
+      if (v != 0 && v != 1 && v != 2 && v != 4 && v != 8 && v != 16 && v != 32)
         return fail(WD_ERR_INVALID_ARG, "group size %lld", (long long)v);
       t->G = int(v);
+      if (v) t->G_used = int(v);
       return WD_OK;
     case WD_OPT_P_MAX:
       if (v < 0 || v > (1 << 26)) return fail(WD_ERR_INVALID_ARG, "p_max %lld", (long long)v);
@@ -1245,6 +1262,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
   if (!t) { fail(WD_ERR_INVALID_ARG, "null table"); return INT64_MIN; }
   switch (opt) {
     case WD_OPT_GROUP_SIZE: return t->G;
+    case WD_OPT_GROUP_SIZE_USED: return t->G_used;
     case WD_OPT_P_MAX: return t->pmax;
     case WD_OPT_BATCH: return int64_t(t->batch);
     case WD_OPT_SERIAL: return t->serial;

@@ -331,3 +331,23 @@ def test_config3_single_gpu_full_size(wd):
         qs = from_dev(q)
     cv, cf = oracle.expected_unique(qs, n, 111, 112)
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
+def test_dynamic_group_size_by_load(wd):
+    # P:245 future work, built: |g| = 0 picks |g| per call from the projected load; the
+    # calls of one table then use different |g| — P:89 says the probe sequence is the same
+    n = 400_000
+    keys, vals = wdgen.unique_keys(n, 121), wdgen.values(n, 122)
+    c = capacity_for(n, 0.99)
+    with wd.Table(c, 1, 0) as t:
+        assert t.get_option(wd.WD_OPT_GROUP_SIZE) == 0
+        t.insert(to_dev(keys[: n // 2]), to_dev(vals[: n // 2]))        # load ~0.5
+        assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == 8
+        t.insert(to_dev(keys[n // 2:]), to_dev(vals[n // 2:]))         # load -> 0.99
+        assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == 16
+        q = wdgen.interleaved_queries(n, 121)
+        ov, of = t.retrieve(to_dev(q))
+        gv, gf = from_dev(ov), of.cpu().numpy()
+        assert t.sync() == 0 and t.size() == n
+    cv, cf = oracle.expected_unique(q, n, 121, 122)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
