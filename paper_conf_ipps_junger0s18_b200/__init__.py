@@ -20,7 +20,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libwarpdrive.so")
+# WD_LIBRARY: measurement hook for A/B runs of two builds (tools/); default is in-tree
+LIB_PATH = os.environ.get("WD_LIBRARY") or os.path.join(_HERE, "libwarpdrive.so")
 
 WD_OK, WD_ERR_INVALID_ARG, WD_ERR_OUT_OF_MEMORY, WD_ERR_CUDA, WD_ERR_NCCL = 0, 1, 2, 3, 4
 WD_ERR_TABLE_FULL, WD_ERR_RESERVED_KEY, WD_ERR_EXCHANGE, WD_ERR_UNSUPPORTED = 5, 6, 7, 8

@@ -36,7 +36,7 @@ def rate(n, G, mode, alpha=0.95, kif=0, reps=5, spl=0):
     return n / (sum(ti) / len(ti)) / 1e6, n / (sum(tq) / len(tq)) / 1e6
 
 
-if __name__ == "__main__" and (len(sys.argv) < 2 or sys.argv[1] not in ("noout", "split")):
+if __name__ == "__main__" and (len(sys.argv) < 2 or sys.argv[1] not in ("noout", "split", "cfg")):
     if len(sys.argv) > 1 and sys.argv[1] == "k":
         lg = int(sys.argv[2]) if len(sys.argv) > 2 else 28
         for G, m, ks in [(4, 1, (2, 4, 8)), (4, 2, (1, 2, 4, 8)), (8, 2, (1, 2, 4)),
@@ -89,3 +89,12 @@ if __name__ == "__main__" and len(sys.argv) > 1 and sys.argv[1] == "split":
         for k in ks:
             i, q = rate(1 << lg, G, 0, kif=k, spl=V)
             print(f"n=2^{lg} G={G} V={V} K={k}: insert {i:6.2f} G/s  query {q:6.2f} G/s", flush=True)
+
+
+if __name__ == "__main__" and len(sys.argv) > 1 and sys.argv[1] == "cfg":
+    # kbench.py cfg <lg> G:V:K ...   (V = 0: auto, K = 0: auto)
+    lg = int(sys.argv[2])
+    for c in sys.argv[3:]:
+        G, V, k = (int(x) for x in c.split(":"))
+        i, q = rate(1 << lg, G, 0, kif=k, spl=V)
+        print(f"n=2^{lg} G={G} V={V} K={k}: insert {i:6.2f} G/s  query {q:6.2f} G/s", flush=True)
