@@ -299,7 +299,18 @@ def main():
         return {"kernel": f"probe_kernel<{name}> (G={G})", "bound": "hbm", "achieved": ach,
                 "peak": hbm, "unit": "GB/s", "frac": ach / hbm, "traffic": None,
                 "bytes_per_op": bpo, "launch_ms": ms,
-                "sectors_per_op": pc["ins_sectors" if name == "insert" else "hit_sectors"]}
+                "sectors_per_op": pc["ins_sectors" if name == "insert" else "hit_sectors"],
+                # HBM moves whole 128-B lines for random accesses (C2): the
+                # same kernel against the replay's distinct lines per op
+                "line_model": line_model(name, ms)}
+
+    def line_model(name, ms):
+        lines = pc.get("ins_lines" if name == "insert" else "hit_lines")
+        if lines is None:
+            return None
+        bpo = (8 + 32 if name == "insert" else 9) + 128 * lines
+        ach = n * bpo / (ms * 1e-3) / 1e9
+        return {"lines_per_op": lines, "bytes_per_op": bpo, "achieved": ach, "frac": ach / hbm}
 
     roofline = roof(dom)
     roofline["peak_source"] = peak_src

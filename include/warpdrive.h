@@ -70,7 +70,8 @@ typedef enum {
  * n_gpus > 1: one shard per device 0..n_gpus-1, keys owned by shard p(k),
  * peer access over NVLink; host input is split into n_gpus contiguous chunks.
  * capacity: total slots c (alpha = n / c).  Each shard gets ceil(c / m) slots,
- * rounded up to a multiple of 4 and to at least 32 (the 32-slot region, Fig. 3 Line 6).
+ * rounded up to a multiple of 4 (sector-aligned region starts, C2) and to at least 32
+ * (the 32-slot region, Fig. 3 Line 6), then until the region count is prime (C13').
  * group_size: |g| in {1,2,4,8,16,32}, or 0 = dynamic by load (see
  * WD_OPT_GROUP_SIZE).  Returns NULL on error (see wd_last_error). */
 wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size);

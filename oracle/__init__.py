@@ -43,7 +43,7 @@ def build(force: bool = False) -> str:
 class _Stats(C.Structure):
     _fields_ = [(n, C.c_uint64) for n in
                 ("ops", "windows", "sectors", "new_keys", "updates", "failures", "found",
-                 "max_windows")]
+                 "max_windows", "lines")]
 
     def as_dict(self):
         return {n: int(getattr(self, n)) for n, _ in self._fields_}
@@ -78,6 +78,8 @@ def lib():
         L.or_replay_rebuild.argtypes = [p, p, u64, C.c_int, u32, u32, C.POINTER(_Stats)]
         L.or_replay_rebuild.restype = None
         L.or_replay_base_seed.argtypes = [u32, u32, u64, u32]; L.or_replay_base_seed.restype = u64
+        L.or_region_align.argtypes = []; L.or_region_align.restype = u64
+        assert L.or_region_align() == REGION_ALIGN
         L.or_map_erase.argtypes = [p, p, p, u64]; L.or_map_erase.restype = u64
         L.or_replay_base.argtypes = [u32, u32, u64]; L.or_replay_base.restype = u64
         L.or_physical_capacity.argtypes = [u64]; L.or_physical_capacity.restype = u64
@@ -197,14 +199,23 @@ def table_scans(T):
 
 # ---------------------------------------------------------------- (6) Fig. 3 replay
 TOMB_WORD = 0xFFFFFFFEFFFFFFFF
+# reading C2: region starts are multiples of 4 slots (one 32-byte sector),
+# for every |g| (the probing scheme must not depend on |g|)
+REGION_ALIGN = 4
+
+
+def n_regions(c: int) -> int:
+    """nb, the number of region starts of a c-slot table (eq. 3's modulus)."""
+    return (int(c) - 32) // REGION_ALIGN + 1
 
 
 class Replay:
-    """Sequential single-group replay of Fig. 3 on a c-slot table (c >= 32, c % 4 == 0)
-    with hash seed `seed` (P:161 translated variants; P:63 rebuild with a distinct one)."""
+    """Sequential single-group replay of Fig. 3 on a c-slot table (c >= 32, c % A == 0,
+    A = REGION_ALIGN) with hash seed `seed` (P:161 translated variants; P:63 rebuild with a
+    distinct one)."""
 
     def __init__(self, capacity: int, group_size: int, p_max: int = 1024, seed: int = 0):
-        assert capacity >= 32 and capacity % 4 == 0
+        assert capacity >= 32 and capacity % REGION_ALIGN == 0
         assert group_size in (1, 2, 4, 8, 16, 32)
         self.c, self.G, self.pmax, self.seed = int(capacity), int(group_size), int(p_max), int(seed)
         self.table = np.full(self.c, np.uint64(0xFFFFFFFFFFFFFFFF), np.uint64)
@@ -246,7 +257,7 @@ class Replay:
 
 def physical_capacity(c: int) -> int:
     """Slots a table of requested capacity c must have so that eq. 3 has full period
-    (nb = (c-32)/4 + 1 prime; reading C13')."""
+    (nb = (c-32)/A + 1 prime, A = REGION_ALIGN; reading C13')."""
     return int(lib().or_physical_capacity(int(c)))
 
 

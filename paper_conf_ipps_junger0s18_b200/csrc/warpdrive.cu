@@ -300,7 +300,7 @@ wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
   s.device = device;
   if (cap == 0) return fail(WD_ERR_INVALID_ARG, "capacity per shard exceeds 4 * 2^32 slots");
   s.cap = cap;
-  s.nb = (cap - 32) / 4 + 1;
+  s.nb = (cap - 32) / wd::kRegionAlign + 1;
   CK(cudaMalloc(&s.slots, cap * sizeof(unsigned long long)));
   CK(cudaMalloc(&s.counters, wd::CNT_N * sizeof(unsigned long long)));
   if (shared_main) {
@@ -912,17 +912,18 @@ bool is_prime(uint64_t x) {
   return true;
 }
 
-// Reading C13': ceil(c/m) slots, rounded up to a multiple of 4 and >= 32,
-// then up until the number of region starts nb = (c-32)/4 + 1 is prime, so eq. 3's
+// Reading C13': ceil(c/m) slots, rounded up to a multiple of A (C2) and
+// >= 32, then up until the number of region starts nb = (c-32)/A + 1 is prime, so eq. 3's
 // double hashing visits every region before repeating.  0 if nb would not fit 32 bits.
 uint64_t shard_cap(uint64_t capacity, int m) {
+  constexpr uint64_t A = wd::kRegionAlign;
   uint64_t c = (capacity + m - 1) / m;
-  c = round_up(std::max<uint64_t>(c, 32), 4);
-  uint64_t nb = (c - 32) / 4 + 1;
+  c = round_up(std::max<uint64_t>(c, 32), A);
+  uint64_t nb = (c - 32) / A + 1;
   if (nb > 1)
     while (!is_prime(nb)) ++nb;
   if (nb >= (1ull << 32)) return 0;
-  return 4 * (nb - 1) + 32;
+  return A * (nb - 1) + 32;
 }
 
 wd_status_t sticky_status(wd_table* t) {

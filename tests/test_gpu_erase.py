@@ -70,7 +70,7 @@ def test_erase_rebuild_serial_layout(wd, G, V):
     c = oracle.physical_capacity(4000)
     keys, vals = wdgen.unique_keys(n, 91), wdgen.values(n, 92)
     er = keys[1::2]
-    r = oracle.Replay(c, G, p_max=(c - 32) // 4 + 1)
+    r = oracle.Replay(c, G, p_max=oracle.n_regions(c))
     r.insert(keys, vals)
     r.erase(er)
     with wd.Table(4000, 1, G) as t:

@@ -165,7 +165,7 @@ def test_edge_cases(wd):
     keys = wdgen.unique_keys(c, 6)
     with wd.Table(1000, 1, 4) as t:
         assert t.capacity() == c
-        t.set_option(wd.WD_OPT_P_MAX, (c - 32) // 4 + 1)
+        t.set_option(wd.WD_OPT_P_MAX, oracle.n_regions(c))
         gv, gf = gpu_roundtrip(t, keys, keys ^ np.uint32(1), keys)
         assert t.sync() == 0 and t.size() == c and np.all(gf == 1)
         assert np.array_equal(gv, keys ^ np.uint32(1))

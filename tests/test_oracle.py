@@ -239,16 +239,18 @@ def test_table_scans_bruteforce():
 def test_replay_single_region_closed_form(G):
     # c = 32: one region, every p maps to base 0, so Fig. 3 scans slots 0..31 left to
     # right: the i-th distinct key lands in slot i after i//G + 1 windows, touching
-    # ceil((i//G + 1) * G / 4) sectors; the 33rd key exhausts p_max regions (Line 26).
+    # ceil((i//G + 1) * G / 4) sectors and ceil((i//G + 1) * G / 16) 128-byte lines; the
+    # 33rd key exhausts p_max regions (Line 26).
     pmax = 3
     r = oracle.Replay(32, G, p_max=pmax)
     keys = wdgen.unique_keys(33, seed=5)
     vals = wdgen.values(33, seed=5)
     for i in range(32):
-        w0, s0 = r.ins.windows, r.ins.sectors
+        w0, s0, l0 = r.ins.windows, r.ins.sectors, r.ins.lines
         r.insert(keys[i:i + 1], vals[i:i + 1])
         assert r.ins.windows - w0 == i // G + 1
         assert r.ins.sectors - s0 == -(-((i // G + 1) * G) // 4)
+        assert r.ins.lines - l0 == -(-((i // G + 1) * G) // 16)
         assert int(r.table[i]) == (int(vals[i]) << 32) | int(keys[i])
     assert r.ins.new_keys == 32 and r.ins.failures == 0
     w0 = r.ins.windows
@@ -262,15 +264,17 @@ def test_replay_single_region_closed_form(G):
 
 
 def test_replay_base_range():
+    A = oracle.REGION_ALIGN
+    assert A == 4                                   # reading C2: sector-aligned starts
     for c in (32, 36, 100, 1000, 1103768, 2**33 + 4):
         for k in (0, 1, 0xDEADBEEF, 0xFFFFFFFE):
             for p in range(0, 50, 7):
                 b = oracle.Replay.base(k, p, c)
-                assert 0 <= b <= c - 32 and b % 4 == 0
+                assert 0 <= b <= c - 32 and b % A == 0
     # bases over many keys cover the whole range [0, c-32] roughly uniformly
     c = 4096
     bs = np.array([oracle.Replay.base(int(k), 0, c) for k in wdgen.unique_keys(20000, 1)])
-    hist = np.bincount(bs // 4, minlength=(c - 32) // 4 + 1)
+    hist = np.bincount(bs // A, minlength=oracle.n_regions(c))
     assert hist.min() >= 1 and hist.max() < 5 * hist.mean()
 
 
@@ -286,15 +290,17 @@ def _isprime(x):
 
 
 def test_physical_capacity_prime_region_count():
-    # C13': c rounded up (multiple of 4, >= 32) until nb = (c-32)/4 + 1 is prime; minimal
+    # C13': c rounded up (multiple of A, >= 32) until nb = (c-32)/A + 1 is prime; minimal
+    A = oracle.REGION_ALIGN
     for c in [1, 31, 32, 33, 36, 40, 64, 100, 1000, 3200, 6321, 1103765, 282563638]:
         cp = oracle.physical_capacity(c)
-        assert cp >= max(c, 32) and cp % 4 == 0
-        nb = (cp - 32) // 4 + 1
+        assert cp >= max(c, 32) and cp % A == 0
+        nb = (cp - 32) // A + 1
+        assert nb == oracle.n_regions(cp)
         assert nb == 1 or _isprime(nb)
-        c4 = max(32, (c + 3) // 4 * 4)
-        for smaller in range(c4, cp, 4):          # no smaller valid capacity
-            nbs = (smaller - 32) // 4 + 1
+        cA = max(32, (c + A - 1) // A * A)
+        for smaller in range(cA, cp, A):          # no smaller valid capacity
+            nbs = (smaller - 32) // A + 1
             assert not (nbs == 1 or _isprime(nbs))
 
 
@@ -302,18 +308,19 @@ def test_physical_capacity_prime_region_count():
 def test_replay_region_sequence_full_period(nb):
     # eq. 3 with a prime number of region starts and a step in [1, nb-1] visits every
     # region exactly once in nb steps, for every key (Knuth's double-hashing condition).
-    c = 4 * (nb - 1) + 32
+    A = oracle.REGION_ALIGN
+    c = A * (nb - 1) + 32
     for k in wdgen.unique_keys(50, nb):
-        seq = [oracle.Replay.base(int(k), p, c) // 4 for p in range(nb)]
+        seq = [oracle.Replay.base(int(k), p, c) // A for p in range(nb)]
         assert sorted(seq) == list(range(nb))
-        assert oracle.Replay.base(int(k), nb, c) == seq[0] * 4   # then it repeats
+        assert oracle.Replay.base(int(k), nb, c) == seq[0] * A   # then it repeats
 
 
 @pytest.mark.parametrize("G", [1, 4, 32])
 def test_replay_fills_table_completely(G):
     # with p_max >= nb every slot is reachable: a table can be filled to alpha = 1
     c = oracle.physical_capacity(400)
-    nb = (c - 32) // 4 + 1
+    nb = oracle.n_regions(c)
     r = oracle.Replay(c, G, p_max=nb)
     keys = wdgen.unique_keys(c + 1, 17)
     r.insert(keys[:c], wdgen.values(c, 17))
@@ -423,7 +430,7 @@ def test_replay_with_tombstones_equals_map(G):
     # them (C9'); results equal the plain dictionary through insert/erase/insert rounds
     n = 4000
     c = oracle.physical_capacity(3 * n)
-    r = oracle.Replay(c, G, p_max=(c - 32) // 4 + 1)
+    r = oracle.Replay(c, G, p_max=oracle.n_regions(c))
     m = oracle.Map(n)
     keys = wdgen.unique_keys(n, 61)
     r.insert(keys, wdgen.values(n, 62)); m.insert(keys, wdgen.values(n, 62))

@@ -1,4 +1,5 @@
-"""Write tests/golden/probe_cost.json: windows and distinct 32-byte sectors per op of the
+"""Write tests/golden/probe_cost.json: windows, distinct 32-byte sectors and distinct
+128-byte lines per op of the
 sequential Fig. 3 replay (oracle only) for alpha x |g|, at n = 2^22 unique keys.
 
 These are the ALGORITHMIC sector counts S of SURVEY §8(d) (the bytes the method must move
@@ -22,7 +23,8 @@ def main(n=1 << 22):
     keys, vals = wdgen.unique_keys(n, 1), wdgen.values(n, 2)
     absent = wdgen.unique_keys(n // 4, 1, start=n)
     out = {"_source": "tools/probe_cost.py: oracle.Replay (sequential Fig. 3, readings C1/C2, "
-                      "sector-aligned 32-slot regions, prime region count), n = %d unique keys, p_max = 1024" % n,
+                      "sector-aligned 32-slot regions (C2), prime region count), "
+                      "n = %d unique keys, p_max = 1024" % n,
            "rows": []}
     for alpha in (0.8, 0.9, 0.95, 0.99):
         c = oracle.physical_capacity(int(math.ceil(n / alpha)))
@@ -38,6 +40,8 @@ def main(n=1 << 22):
                    "hit_windows": st_hit.windows / st_hit.ops, "hit_sectors": st_hit.sectors / st_hit.ops,
                    "miss_windows": st_miss.windows / st_miss.ops,
                    "miss_sectors": st_miss.sectors / st_miss.ops,
+                   "ins_lines": r.ins.lines / n, "hit_lines": st_hit.lines / st_hit.ops,
+                   "miss_lines": st_miss.lines / st_miss.ops,
                    "max_ins_windows": int(r.ins.max_windows)}
             out["rows"].append(row)
             print(row, flush=True)
