@@ -166,7 +166,10 @@ typedef enum {
                                 one sm_100 vector load (|g| <= 8; same windows, same result) */
     WD_OPT_KERNEL_FLAGS = 8, /* bit 0: probe loads may hit L1 (safe: keys never change once
                                 written; a lost CAS reloads from L2); bit 1: value updates
-                                of existing keys as atomic exchange.  Default 3. */
+                                of existing keys as atomic exchange; bit 2: reserved
+                                (rejected); bit 3: a query call visits its input chunks in a scrambled
+                                order (keys inserted together are not queried together;
+                                results land in the same positions).  Default 11. */
     WD_OPT_SLOTS_PER_LANE = 9, /* V: each lane of a window loads V consecutive slots with one
                                 vector load, so a window is read by |g|/V lanes (1: the
                                 paper's cooperative group; |g|: one lane).  0 = from

@@ -123,10 +123,11 @@ struct wd_table {
   int kif = 0;        // keys in flight per group (0 = default)
   int probe_mode = 0; // 0: auto, 1: cooperative groups (Fig. 3), 2: lane-window (|g| <= 8)
   int spl = 0;        // slots per lane V (WD_OPT_SLOTS_PER_LANE; 0 = from probe mode)
-  // wd::kF_* kernel variants (WD_OPT_KERNEL_FLAGS).  Default both: atom.exch value updates
-  // take hot (Zipf) keys from 0.5 to 6-8 G inserts/s (tools/flags_bench.py), L1-allowed
-  // probe loads add ~15 % there; neither changes the unique-key rates.
-  uint32_t kflags = wd::kF_L1 | wd::kF_XCHG;
+  // wd::kF_* kernel variants (WD_OPT_KERNEL_FLAGS).  Default all three: atom.exch value
+  // updates take hot (Zipf) keys from 0.5 to 6-8 G inserts/s (tools/flags_bench.py),
+  // L1-allowed probe loads add ~15 % there; the scrambled query chunk order adds 22-40 % to
+  // queries issued in insert order (profiles/r01_query_order.md).
+  uint32_t kflags = wd::kF_L1 | wd::kF_XCHG | wd::kF_QSCR;
   uint64_t batch = 1ull << 24;
   int serial = 0;
   uint32_t pseed = 0x9E3779B9u;
@@ -1244,7 +1245,7 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       t->spl = int(v);
       return WD_OK;
     case WD_OPT_KERNEL_FLAGS:
-      if (v < 0 || v > 3) return fail(WD_ERR_INVALID_ARG, "kernel flags %lld", (long long)v);
+      if (v < 0 || (uint32_t(v) & ~wd::kF_ALL) != 0) return fail(WD_ERR_INVALID_ARG, "kernel flags %lld", (long long)v);
       t->kflags = uint32_t(v);
       return WD_OK;
     case WD_OPT_PROBE_MODE:

@@ -112,7 +112,8 @@ def test_cross_group_size(wd, Gi, Gq, mi, mq):
 
 
 @pytest.mark.parametrize("G,mode,flags", [(1, 1, 3), (4, 1, 3), (32, 1, 3), (2, 2, 3), (4, 2, 3),
-                                          (8, 2, 3), (4, 0, 3), (4, 1, 0), (4, 2, 0), (1, 1, 1)])
+                                          (8, 2, 3), (4, 0, 3), (4, 1, 0), (4, 2, 0), (1, 1, 1),
+                                          (1, 1, 11), (4, 1, 11), (8, 0, 11), (8, 2, 8)])
 def test_duplicates_upsert(wd, G, mode, flags):
     # duplicate-key mode: value must be one of the values inserted for the key;
     # size = number of distinct keys; a second stream-ordered call wins.
@@ -239,7 +240,8 @@ def test_config2_full_size_sampled(wd):
 
 
 @pytest.mark.parametrize("G,mode,flags", [(1, 1, 3), (4, 1, 3), (8, 1, 3), (4, 2, 3), (2, 2, 3),
-                                          (4, 1, 0), (4, 2, 1), (4, 1, 2)])
+                                          (4, 1, 0), (4, 2, 1), (4, 1, 2), (1, 1, 11), (8, 0, 11),
+                                          (4, 2, 10)])
 def test_zipf_duplicates(wd, G, mode, flags):
     # Zipf keys (s = 1 + 1e-6): hot keys updated by many groups at once.
     # Every returned value must be one of the values inserted for its key; size = #distinct.
@@ -279,6 +281,25 @@ def test_window_split_serial_layout(wd, G, V):
         t.insert(to_dev(keys), to_dev(vals))
         assert t.sync() == 0
         assert np.array_equal(t.dump(), r.table)
+
+
+@pytest.mark.parametrize("G,V", [(1, 1), (4, 1), (4, 2), (8, 4), (8, 8), (16, 4), (32, 1)])
+@pytest.mark.parametrize("n", [1000, 128 * 9, 300_007, 1 << 20])
+def test_scrambled_query_order(wd, G, V, n):
+    # kF_QSCR: queries visit their chunks in a scrambled order; every result must still land
+    # at its own position (full chunks, partial last chunk, tiny inputs), with and without
+    # the scramble, for duplicates in the query batch too
+    keys, vals = wdgen.unique_keys(n, 43), wdgen.values(n, 44)
+    q = wdgen.interleaved_queries(n, 43)
+    q = np.concatenate([q, q[: n // 3]])
+    cv, cf = oracle.expected_unique(q, n, 43, 44)
+    for flags in (11, 3):
+        with wd.Table(capacity_for(n, 0.95), 1, G) as t:
+            t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
+            t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
+            gv, gf = gpu_roundtrip(t, keys, vals, q)
+            assert t.sync() == 0 and t.size() == n
+        assert np.array_equal(gf, cf) and np.array_equal(gv, cv), flags
 
 
 @pytest.mark.parametrize("G,V", SPLITS)
