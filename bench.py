@@ -152,6 +152,17 @@ def cpu_baseline_sample(log2n: int = 26):
             "seconds": t2 - t0, "host_cpus": os.cpu_count()}
 
 
+def workload_config(args, world):
+    n = 1 << args.n_log2
+    return {"workload": f"config2: 2^{args.n_log2} unique u32 key/value pairs per GPU, "
+                        f"load {args.alpha}, |g|={args.group_size}; step = fill + insert all + "
+                        f"retrieve all (100% hits, queried in insert order)",
+            "global_batch": n * world, "pairs_per_gpu": n, "alpha": args.alpha,
+            "group_size": args.group_size,
+            "parallelism": f"keyspace-shard{world}" if world > 1 else "single",
+            "l2": "inputs (2 x 2^%d x 4 B) and table exceed the 126 MB L2; no flush" % args.n_log2}
+
+
 # ----------------------------------------------------------------------------- reference arm
 def run_reference(args):
     """--impl reference: the oracle (this tier's reference arm) on the host cores, on the
@@ -180,9 +191,9 @@ def run_reference(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic", "impl": "reference",
-            "config": {"workload": "config2: 2^28 unique u32 pairs, alpha 0.95, |g| 4, "
-                                   "insert + retrieve (reference arm: bounded 2^22 sample per step)",
-                       "global_batch": n, "alpha": args.alpha, "group_size": args.group_size},
+            "config": dict(workload_config(args, args.gpus),
+                           reference_sample="bounded 2^22 unique inserts + 2^22 hit queries "
+                                            "per step, single-threaded C oracle"),
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
                              "sample": "2^22 unique inserts + 2^22 hit queries per step"},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -368,13 +379,8 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_ms,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u32", "data": "synthetic",
-            "config": {"workload": f"config2: 2^{args.n_log2} unique u32 key/value pairs per GPU, "
-                                   f"load {args.alpha}, |g|={G}; step = fill + insert all + "
-                                   f"retrieve all (100% hits)",
-                       "global_batch": n * world, "pairs_per_gpu": n, "alpha": args.alpha,
-                       "group_size": G, "capacity_per_gpu": table.shard_capacity(0),
-                       "parallelism": f"keyspace-shard{world}" if world > 1 else "single",
-                       "l2": "inputs (2 x 2^%d x 4 B) and table exceed the 126 MB L2; no flush" % args.n_log2},
+            "config": dict(workload_config(args, world),
+                           capacity_per_gpu=table.shard_capacity(0)),
             "insert_gops": n * world / (ins_ms * 1e-3) / 1e9,
             "query_gops": n * world / (qry_ms * 1e-3) / 1e9,
             "fill_ms": t_ms - ins_ms - qry_ms,
@@ -424,8 +430,102 @@ def run_sweep(args, wd, gg, torch):
                             "insert_gops": n / ims / 1e6, "query_gops": n / qms / 1e6,
                             "insert_frac": n * (40 + 32 * pc["ins_sectors"]) / (ims * 1e-3) / 1e9 / hbm,
                             "query_frac": n * (9 + 32 * pc["hit_sectors"]) / (qms * 1e-3) / 1e9 / hbm})
+    out += run_mix(wd, gg, torch, keys, vals, args.n_log2)
     del keys, vals, vout, fout
     out += run_zipf(wd, gg, torch)
+    out += run_ooc(wd, gg, torch)
+    return out
+
+
+def run_mix(wd, gg, torch, keys, vals, log2n):
+    """BASELINE config 4 at one GPU: a 2^log2n-key table at alpha 0.95, then 2^log2n queries
+    with hit fraction 0 / 0.5 / 1 (wdgen.mixed_queries: a hit is a stored key, a miss a key
+    never inserted).  found must equal the generator's hit flag for every query."""
+    out = []
+    n = 1 << log2n
+    q = torch.empty(n, dtype=torch.int32, device="cuda")
+    hits = torch.empty(n, dtype=torch.uint8, device="cuda")
+    vout = torch.empty(n, dtype=torch.int32, device="cuda")
+    fout = torch.empty(n, dtype=torch.uint8, device="cuda")
+    s = torch.cuda.current_stream()
+    hbm, _ = peaks()
+    for G in (4, 8, 16):
+        with wd.Table(int(math.ceil(n / 0.95)), 1, G) as t:
+            t.insert(keys, vals, s)
+            for h in (0.0, 0.5, 1.0):
+                gg.mixed_queries(n, n, h, KEY_SEED, out=q, hits=hits)
+                ts = []
+                for it in range(4):
+                    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record(s)
+                    t.retrieve(q, vout, fout, s)
+                    b.record(s)
+                    torch.cuda.synchronize()
+                    if it:
+                        ts.append(a.elapsed_time(b))
+                assert t.sync() == 0 and bool((fout == hits).all())
+                ms = sum(ts) / len(ts)
+                pc = probe_cost(0.95, G)
+                S = h * pc["hit_sectors"] + (1 - h) * pc["miss_sectors"]
+                out.append({"sweep": "config4_mix_1gpu", "alpha": 0.95, "G": G, "hit_frac": h,
+                            "table_keys": n, "queries": n, "query_gops": n / ms / 1e6,
+                            "sectors_per_query": S,
+                            "query_frac": n * (9 + 32 * S) / (ms * 1e-3) / 1e9 / hbm})
+    return out
+
+
+def run_ooc(wd, gg, torch, log2n=30):
+    """BASELINE config 5 scaled to one GPU: 2^log2n uniform draws WITH replacement (duplicate
+    keys) in pinned host memory, streamed through the C-ABI's out-of-core pipeline
+    (H2D(b+1) || insert(b), batches of 2^24 pairs) into a table sized for the expected
+    number of distinct keys at alpha 0.95 (C13); then all draws are queried back to pinned
+    host memory.  Checks: size = distinct count; every query found; on the keys with
+    k mod 1024 == 0, each returned value is one of the values drawn for that key."""
+    n = 1 << log2n
+    keys = gg.uniform_keys(n, KEY_SEED)
+    vals = gg.values(n, VAL_SEED)
+    distinct = int(torch.unique(keys).numel())
+    expect = 2**32 * (1 - math.exp(-n / 2**32))
+    hk = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    hv = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    hk.copy_(keys)
+    hv.copy_(vals)
+    hvo = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    hfo = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+    s = torch.cuda.current_stream()
+    out = []
+    with wd.Table(int(math.ceil(expect / 0.95)), 1, 8, batch=1 << 24) as t:
+        ti, tq = [], []
+        for it in range(3):
+            a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            t.clear(s)
+            a.record(s)
+            t.insert(hk, hv, s)
+            b.record(s)
+            t.retrieve(hk, hvo, hfo, s)
+            c.record(s)
+            torch.cuda.synchronize()
+            if it:
+                ti.append(a.elapsed_time(b))
+                tq.append(b.elapsed_time(c))
+        assert t.sync() == 0 and t.size() == distinct
+        assert bool((hfo == 1).all())
+        # subset check of duplicate mode: (k, returned v) must be a drawn pair
+        sel = (keys.to(torch.int64) & 0xFFFFFFFF) % 1024 == 0
+        pairs = ((keys[sel].to(torch.int64) & 0xFFFFFFFF) << 32) | (vals[sel].to(torch.int64) & 0xFFFFFFFF)
+        pairs = torch.unique(pairs)
+        got = ((keys[sel].to(torch.int64) & 0xFFFFFFFF) << 32) | \
+              (hvo.cuda()[sel].to(torch.int64) & 0xFFFFFFFF)
+        pos = torch.searchsorted(pairs, got).clamp(max=pairs.numel() - 1)
+        assert bool((pairs[pos] == got).all()), "duplicate mode: value not among the drawn ones"
+        ims, qms = sum(ti) / len(ti), sum(tq) / len(tq)
+        out.append({"sweep": "config5_ooc_1gpu", "draws": n, "distinct": distinct,
+                    "expected_distinct": expect, "alpha_actual": distinct / t.capacity(),
+                    "G": 8, "batch": 1 << 24, "insert_gops_e2e": n / ims / 1e6,
+                    "query_gops_e2e": n / qms / 1e6,
+                    "h2d_GBps_insert": 8 * n / (ims * 1e-3) / 1e9,
+                    "pcie_bytes": {"insert_h2d": 8 * n, "query_h2d": 4 * n, "query_d2h": 5 * n},
+                    "checked_pairs": int(sel.sum().item())})
     return out
 
 

@@ -275,6 +275,10 @@ wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, 
 template <bool INSERT, class In, class Out>
 wd_status_t launch_probe(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                          cudaStream_t st) {
+#ifdef WD_ONLY_G   // experiment builds (tools/ab_lib.sh): one group size, a fraction of the build time
+  if (t->G_used == WD_ONLY_G) return launch_probe_g<WD_ONLY_G, INSERT>(t, s, in, out, n_hint, st);
+  return fail(WD_ERR_UNSUPPORTED, "experiment build: only |g| = %d", WD_ONLY_G);
+#endif
   switch (t->G_used) {
     case 1: return launch_probe_g<1, INSERT>(t, s, in, out, n_hint, st);
     case 2: return launch_probe_g<2, INSERT>(t, s, in, out, n_hint, st);
