@@ -70,19 +70,21 @@ def lib():
         L.or_multisplit.argtypes = [p, u64, u32, u32, C.c_int, p, p]
         L.or_multisplit.restype = None
         L.or_table_scans.argtypes = [p, u32, p, p]; L.or_table_scans.restype = None
-        L.or_replay_insert.argtypes = [p, u64, C.c_int, u32, u32, p, p, u64, C.POINTER(_Stats)]
+        L.or_replay_insert.argtypes = [p, u64, u32, C.c_int, u32, u32, p, p, u64, C.POINTER(_Stats)]
         L.or_replay_insert.restype = None
-        L.or_replay_query.argtypes = [p, u64, C.c_int, u32, u32, p, p, p, u64,
+        L.or_replay_query.argtypes = [p, u64, u32, C.c_int, u32, u32, p, p, p, u64,
                                       C.POINTER(_Stats), C.c_int]
         L.or_replay_query.restype = None
-        L.or_replay_rebuild.argtypes = [p, p, u64, C.c_int, u32, u32, C.POINTER(_Stats)]
+        L.or_replay_rebuild.argtypes = [p, p, u64, u32, C.c_int, u32, u32, C.POINTER(_Stats)]
         L.or_replay_rebuild.restype = None
-        L.or_replay_base_seed.argtypes = [u32, u32, u64, u32]; L.or_replay_base_seed.restype = u64
+        L.or_replay_base_seed.argtypes = [u32, u32, u64, u32, u32]
+        L.or_replay_base_seed.restype = u64
         L.or_region_align.argtypes = []; L.or_region_align.restype = u64
         assert L.or_region_align() == REGION_ALIGN
         L.or_map_erase.argtypes = [p, p, p, u64]; L.or_map_erase.restype = u64
         L.or_replay_base.argtypes = [u32, u32, u64]; L.or_replay_base.restype = u64
         L.or_physical_capacity.argtypes = [u64]; L.or_physical_capacity.restype = u64
+        L.or_physical_capacity_a.argtypes = [u64, u64]; L.or_physical_capacity_a.restype = u64
         for f in (L.or_fmix32_many, L.or_mueller_many):
             f.argtypes = [p, p, u64]; f.restype = None
         L.or_partition_many.argtypes = [p, p, u64, u32, u32, C.c_int]
@@ -199,32 +201,43 @@ def table_scans(T):
 
 # ---------------------------------------------------------------- (6) Fig. 3 replay
 TOMB_WORD = 0xFFFFFFFEFFFFFFFF
-# reading C2: region starts are multiples of 4 slots (one 32-byte sector),
-# for every |g| (the probing scheme must not depend on |g|)
+# reading C2': region starts are multiples of A slots, A a property of the
+# table, the same for every |g| used on it (the probing scheme must not depend on |g|):
+# A = 4 (one 32-byte sector) by default, A = 16 (one 128-byte line) for a table created
+# with |g| >= 16, so that its 128-byte windows never straddle two lines
 REGION_ALIGN = 4
+LINE_ALIGN = 16
 
 
-def n_regions(c: int) -> int:
+def region_align_for(group_size: int) -> int:
+    """A of a table created with |g| = group_size (0 = dynamic |g|: the default A)."""
+    return LINE_ALIGN if int(group_size) >= 16 else REGION_ALIGN
+
+
+def n_regions(c: int, align: int = REGION_ALIGN) -> int:
     """nb, the number of region starts of a c-slot table (eq. 3's modulus)."""
-    return (int(c) - 32) // REGION_ALIGN + 1
+    return (int(c) - 32) // int(align) + 1
 
 
 class Replay:
     """Sequential single-group replay of Fig. 3 on a c-slot table (c >= 32, c % A == 0,
-    A = REGION_ALIGN) with hash seed `seed` (P:161 translated variants; P:63 rebuild with a
+    A = align) with hash seed `seed` (P:161 translated variants; P:63 rebuild with a
     distinct one)."""
 
-    def __init__(self, capacity: int, group_size: int, p_max: int = 1024, seed: int = 0):
-        assert capacity >= 32 and capacity % REGION_ALIGN == 0
+    def __init__(self, capacity: int, group_size: int, p_max: int = 1024, seed: int = 0,
+                 align: int = REGION_ALIGN):
+        assert align in (REGION_ALIGN, LINE_ALIGN)
+        assert capacity >= 32 and capacity % align == 0
         assert group_size in (1, 2, 4, 8, 16, 32)
         self.c, self.G, self.pmax, self.seed = int(capacity), int(group_size), int(p_max), int(seed)
+        self.align = int(align)
         self.table = np.full(self.c, np.uint64(0xFFFFFFFFFFFFFFFF), np.uint64)
         self.ins = _Stats()
         self.qry = _Stats()
 
     def insert(self, keys, vals):
         k, v = _u32(keys), _u32(vals)
-        lib().or_replay_insert(_ptr(self.table), self.c, self.G, self.pmax, self.seed, _ptr(k),
+        lib().or_replay_insert(_ptr(self.table), self.c, self.align, self.G, self.pmax, self.seed, _ptr(k),
                                _ptr(v), k.size, C.byref(self.ins))
 
     def query(self, keys, stats: _Stats | None = None, erase: bool = False):
@@ -232,7 +245,7 @@ class Replay:
         vals = np.empty(k.size, np.uint32)
         found = np.empty(k.size, np.uint8)
         st = stats if stats is not None else self.qry
-        lib().or_replay_query(_ptr(self.table), self.c, self.G, self.pmax, self.seed, _ptr(k),
+        lib().or_replay_query(_ptr(self.table), self.c, self.align, self.G, self.pmax, self.seed, _ptr(k),
                               _ptr(vals), _ptr(found), k.size, C.byref(st), int(erase))
         return vals, found
 
@@ -246,19 +259,19 @@ class Replay:
         self.seed = int(seed)
         self.table = np.full(self.c, np.uint64(0xFFFFFFFFFFFFFFFF), np.uint64)
         st = _Stats()
-        lib().or_replay_rebuild(_ptr(old), _ptr(self.table), self.c, self.G, self.pmax,
+        lib().or_replay_rebuild(_ptr(old), _ptr(self.table), self.c, self.align, self.G, self.pmax,
                                 self.seed, C.byref(st))
         return st
 
     @staticmethod
-    def base(k: int, p: int, capacity: int, seed: int = 0) -> int:
-        return int(lib().or_replay_base_seed(int(k), int(p), int(capacity), int(seed)))
+    def base(k: int, p: int, capacity: int, seed: int = 0, align: int = REGION_ALIGN) -> int:
+        return int(lib().or_replay_base_seed(int(k), int(p), int(capacity), int(seed), int(align)))
 
 
-def physical_capacity(c: int) -> int:
+def physical_capacity(c: int, align: int = REGION_ALIGN) -> int:
     """Slots a table of requested capacity c must have so that eq. 3 has full period
-    (nb = (c-32)/A + 1 prime, A = REGION_ALIGN; reading C13')."""
-    return int(lib().or_physical_capacity(int(c)))
+    (nb = (c-32)/A + 1 prime, A = align; reading C13')."""
+    return int(lib().or_physical_capacity_a(int(c), int(align)))
 
 
 # ---------------------------------------------------------------- closed form (generator)

@@ -263,18 +263,21 @@ def test_replay_single_region_closed_form(G):
     assert np.all(f == 1) and np.array_equal(v, vals[:32])
 
 
-def test_replay_base_range():
-    A = oracle.REGION_ALIGN
-    assert A == 4                                   # reading C2: sector-aligned starts
-    for c in (32, 36, 100, 1000, 1103768, 2**33 + 4):
+@pytest.mark.parametrize("A", [4, 16])
+def test_replay_base_range(A):
+    # reading C2': sector-aligned starts (A = 4), line-aligned for |g| >= 16 tables (A = 16)
+    assert oracle.REGION_ALIGN == 4 and oracle.LINE_ALIGN == 16
+    assert oracle.region_align_for(8) == 4 and oracle.region_align_for(16) == 16
+    assert oracle.region_align_for(0) == 4
+    for c in (32, 48, 112, 1008, 1103776, 2**33 + 16):
         for k in (0, 1, 0xDEADBEEF, 0xFFFFFFFE):
             for p in range(0, 50, 7):
-                b = oracle.Replay.base(k, p, c)
+                b = oracle.Replay.base(k, p, c, align=A)
                 assert 0 <= b <= c - 32 and b % A == 0
     # bases over many keys cover the whole range [0, c-32] roughly uniformly
-    c = 4096
-    bs = np.array([oracle.Replay.base(int(k), 0, c) for k in wdgen.unique_keys(20000, 1)])
-    hist = np.bincount(bs // A, minlength=oracle.n_regions(c))
+    c = 4096 if A == 4 else 16384
+    bs = np.array([oracle.Replay.base(int(k), 0, c, align=A) for k in wdgen.unique_keys(20000, 1)])
+    hist = np.bincount(bs // A, minlength=oracle.n_regions(c, A))
     assert hist.min() >= 1 and hist.max() < 5 * hist.mean()
 
 
@@ -289,14 +292,16 @@ def _isprime(x):
     return True
 
 
-def test_physical_capacity_prime_region_count():
+@pytest.mark.parametrize("A", [4, 16])
+def test_physical_capacity_prime_region_count(A):
     # C13': c rounded up (multiple of A, >= 32) until nb = (c-32)/A + 1 is prime; minimal
-    A = oracle.REGION_ALIGN
+    if A == 4:
+        assert oracle.physical_capacity(1000) == oracle.physical_capacity(1000, 4)
     for c in [1, 31, 32, 33, 36, 40, 64, 100, 1000, 3200, 6321, 1103765, 282563638]:
-        cp = oracle.physical_capacity(c)
+        cp = oracle.physical_capacity(c, A)
         assert cp >= max(c, 32) and cp % A == 0
         nb = (cp - 32) // A + 1
-        assert nb == oracle.n_regions(cp)
+        assert nb == oracle.n_regions(cp, A)
         assert nb == 1 or _isprime(nb)
         cA = max(32, (c + A - 1) // A * A)
         for smaller in range(cA, cp, A):          # no smaller valid capacity
@@ -304,24 +309,25 @@ def test_physical_capacity_prime_region_count():
             assert not (nbs == 1 or _isprime(nbs))
 
 
+@pytest.mark.parametrize("A", [4, 16])
 @pytest.mark.parametrize("nb", [2, 3, 13, 101, 1009])
-def test_replay_region_sequence_full_period(nb):
+def test_replay_region_sequence_full_period(nb, A):
     # eq. 3 with a prime number of region starts and a step in [1, nb-1] visits every
     # region exactly once in nb steps, for every key (Knuth's double-hashing condition).
-    A = oracle.REGION_ALIGN
     c = A * (nb - 1) + 32
     for k in wdgen.unique_keys(50, nb):
-        seq = [oracle.Replay.base(int(k), p, c) // A for p in range(nb)]
+        seq = [oracle.Replay.base(int(k), p, c, align=A) // A for p in range(nb)]
         assert sorted(seq) == list(range(nb))
-        assert oracle.Replay.base(int(k), nb, c) == seq[0] * A   # then it repeats
+        assert oracle.Replay.base(int(k), nb, c, align=A) == seq[0] * A   # then it repeats
 
 
+@pytest.mark.parametrize("A", [4, 16])
 @pytest.mark.parametrize("G", [1, 4, 32])
-def test_replay_fills_table_completely(G):
+def test_replay_fills_table_completely(G, A):
     # with p_max >= nb every slot is reachable: a table can be filled to alpha = 1
-    c = oracle.physical_capacity(400)
-    nb = oracle.n_regions(c)
-    r = oracle.Replay(c, G, p_max=nb)
+    c = oracle.physical_capacity(400, A)
+    nb = oracle.n_regions(c, A)
+    r = oracle.Replay(c, G, p_max=nb, align=A)
     keys = wdgen.unique_keys(c + 1, 17)
     r.insert(keys[:c], wdgen.values(c, 17))
     assert r.ins.new_keys == c and r.ins.failures == 0
@@ -330,15 +336,17 @@ def test_replay_fills_table_completely(G):
     assert r.ins.failures == 1
 
 
-def test_replay_layout_independent_of_group_size_p89():
+@pytest.mark.parametrize("A", [4, 16])
+def test_replay_layout_independent_of_group_size_p89(A):
     # "The inner probing loop (Line 6) ensures a consistent probing scheme in case
-    # that the size of g is varied": the sequential layout must not depend on |g|.
+    # that the size of g is varied": the sequential layout must not depend on |g| — for a
+    # given table geometry (A is a property of the table, reading C2').
     n, c = 6000, 6320
     keys = wdgen.unique_keys(n, 8)
     vals = wdgen.values(n, 8)
     tables = []
     for G in (1, 2, 4, 8, 16, 32):
-        r = oracle.Replay(c, G)
+        r = oracle.Replay(c, G, align=A)
         r.insert(keys, vals)
         assert r.ins.new_keys == n
         tables.append(r.table.copy())
@@ -346,18 +354,19 @@ def test_replay_layout_independent_of_group_size_p89():
         assert np.array_equal(t, tables[0])
 
 
+@pytest.mark.parametrize("A,G", [(4, 4), (16, 16), (16, 4)])
 @pytest.mark.parametrize("dup", [False, True])
-def test_replay_results_equal_map(dup):
+def test_replay_results_equal_map(dup, A, G):
     # the replay of Fig. 3 reaches the same map as the plain dictionary (sequential
     # upserts, last value wins), for hits, misses and updates
     n = 20000
-    c = oracle.physical_capacity(int(n / 0.95))
+    c = oracle.physical_capacity(int(n / 0.95), A)
     if dup:
         keys = wdgen.uniform_keys(n, 3) % np.uint32(9000)  # many repeats
     else:
         keys = wdgen.unique_keys(n, 3)
     vals = wdgen.values(n, 4)
-    r = oracle.Replay(c, 4)
+    r = oracle.Replay(c, G, align=A)
     r.insert(keys, vals)
     m = oracle.Map(n)
     m.insert(keys, vals)
@@ -366,6 +375,24 @@ def test_replay_results_equal_map(dup):
     rv, rf = r.query(q)
     mv, mf = m.retrieve(q)
     assert np.array_equal(rf, mf) and np.array_equal(rv, mv)
+
+
+def test_replay_line_aligned_windows_touch_one_line():
+    # A = 16: a 128-byte window (|g| = 16) starts on a line boundary, so every window the
+    # replay counts is exactly one distinct 128-byte line and four sectors (and with A = 4
+    # most windows straddle two lines) — pins that the alignment reaches Line 7's address
+    n = 1 << 14
+    keys, vals = wdgen.unique_keys(n, 21), wdgen.values(n, 21)
+    c16 = oracle.physical_capacity(int(n / 0.95), 16)
+    r = oracle.Replay(c16, 16, align=16)
+    r.insert(keys, vals)
+    assert r.ins.lines == r.ins.windows and r.ins.sectors == 4 * r.ins.windows
+    _, f = r.query(keys)
+    assert np.all(f == 1) and r.qry.lines == r.qry.windows
+    c4 = oracle.physical_capacity(int(n / 0.95), 4)
+    r4 = oracle.Replay(c4, 16)
+    r4.insert(keys, vals)
+    assert r4.ins.lines > 1.5 * r4.ins.windows
 
 
 def test_replay_probe_costs_grow_with_load():

@@ -23,19 +23,22 @@ def main(n=1 << 22):
     keys, vals = wdgen.unique_keys(n, 1), wdgen.values(n, 2)
     absent = wdgen.unique_keys(n // 4, 1, start=n)
     out = {"_source": "tools/probe_cost.py: oracle.Replay (sequential Fig. 3, readings C1/C2, "
-                      "sector-aligned 32-slot regions (C2), prime region count), "
+                      "32-slot regions starting at multiples of A = 4 slots, A = 16 for |g| >= 16 (C2'), "
+                      "prime region count), "
                       "n = %d unique keys, p_max = 1024" % n,
            "rows": []}
     for alpha in (0.8, 0.9, 0.95, 0.99):
         c = oracle.physical_capacity(int(math.ceil(n / alpha)))
         for G in (1, 2, 4, 8, 16, 32):
-            r = oracle.Replay(c, G)
+            A = oracle.region_align_for(G)      # the geometry the library gives a |g| table
+            c = oracle.physical_capacity(int(math.ceil(n / alpha)), A)
+            r = oracle.Replay(c, G, align=A)
             r.insert(keys, vals)
             st_hit = oracle._Stats()
             r.query(keys[::4], st_hit)  # spread over insertion order
             st_miss = oracle._Stats()
             r.query(absent, st_miss)
-            row = {"alpha": alpha, "G": G,
+            row = {"alpha": alpha, "G": G, "align": A,
                    "ins_windows": r.ins.windows / n, "ins_sectors": r.ins.sectors / n,
                    "hit_windows": st_hit.windows / st_hit.ops, "hit_sectors": st_hit.sectors / st_hit.ops,
                    "miss_windows": st_miss.windows / st_miss.ops,
