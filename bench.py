@@ -5,7 +5,7 @@
 
 One step = one pass of the whole hot path over one batch of synthetic input
 (SURVEY §8(a)): a1 table fill, a2+a3 insert of n unique pairs, a2+a4 retrieve of the same
-n keys (100 % hits; BASELINE config 2's "insert and retrieve" at alpha = 0.95, |g| = 4);
+n keys (100 % hits; BASELINE config 2's "insert and retrieve" at alpha = 0.95, |g| = 16);
 with N > 1 (torchrun, one process per GPU, weak scaling: n pairs per GPU) the insert and
 retrieve run the distributed cascades a6-a10 (multisplit fused with the NVLink push, T
 flags, local probe, reverse pull + unpermute).
@@ -49,8 +49,9 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--n-log2", type=int, default=28, help="pairs per GPU (config 2: 28)")
     ap.add_argument("--alpha", type=float, default=0.95)
-    ap.add_argument("--group-size", type=int, default=8,
-                    help="|g| (config 2 sweeps 1-32; 8 is the fastest at alpha 0.95 on B200)")
+    ap.add_argument("--group-size", type=int, default=16,
+                    help="|g| (config 2 sweeps 1-32; 16 is the fastest at alpha 0.95 on B200, "
+                         "profiles/r01_sweep.jsonl)")
     ap.add_argument("--kif", type=int, default=0, help="keys in flight per group (0=default)")
     ap.add_argument("--probe-mode", type=int, default=None,
                     help="0: auto; 1: cooperative group per window (Fig. 3); 2: lane-window")

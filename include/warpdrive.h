@@ -70,8 +70,9 @@ typedef enum {
  * n_gpus > 1: one shard per device 0..n_gpus-1, keys owned by shard p(k),
  * peer access over NVLink; host input is split into n_gpus contiguous chunks.
  * capacity: total slots c (alpha = n / c).  Each shard gets ceil(c / m) slots,
- * rounded up to a multiple of 4 (sector-aligned region starts, C2) and to at least 32
- * (the 32-slot region, Fig. 3 Line 6), then until the region count is prime (C13').
+ * rounded up to a multiple of A and to at least 32 (the 32-slot region, Fig. 3 Line 6), then
+ * until the region count is prime (C13').  A = the region-start alignment (C2'):
+ * 16 slots (one 128-byte line) if group_size >= 16, else 4 (one sector).
  * group_size: |g| in {1,2,4,8,16,32}, or 0 = dynamic by load (see
  * WD_OPT_GROUP_SIZE).  Returns NULL on error (see wd_last_error). */
 wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size);
@@ -150,7 +151,7 @@ wd_status_t wd_sync(wd_table_t* t);
 typedef enum {
     WD_OPT_GROUP_SIZE = 0,   /* |g|; the probe sequence does not depend on it.
                                 0 = dynamic by load: 8, or 16 above a projected
-                                load of 0.97 (measured on B200) */
+                                load of 0.93 (measured on B200) */
     WD_OPT_P_MAX = 1,        /* outer probing bound p_max (Fig. 3 Line 4); 0 (default) = the
                                 number of regions nb, i.e. fail only when the table is full (C4') */
     WD_OPT_BATCH = 2,        /* items per shard per pipeline batch (2^24) */
@@ -178,7 +179,12 @@ typedef enum {
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */
     WD_OPT_LAUNCHES = 103,   /* read-only: kernels launched by the library so far */
-    WD_OPT_GROUP_SIZE_USED = 104 /* read-only: |g| used by the last call */
+    WD_OPT_GROUP_SIZE_USED = 104, /* read-only: |g| used by the last call */
+    WD_OPT_REGION_ALIGN = 105  /* read-only: A, region starts are multiples of A slots
+                                  (reading C2'): 16 (one 128-byte line) when the table was
+                                  created with group_size >= 16, else 4 (one sector); fixed
+                                  for the table's life, so every |g| later used on it probes
+                                  the same sequence */
 } wd_option_t;
 
 wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t value);

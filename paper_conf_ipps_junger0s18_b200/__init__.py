@@ -33,6 +33,7 @@ WD_OPT_KEYS_IN_FLIGHT, WD_OPT_PART_SEED, WD_OPT_PART_MODE, WD_OPT_PROBE_MODE = 4
 WD_OPT_KERNEL_FLAGS, WD_OPT_SLOTS_PER_LANE = 8, 9
 WD_OPT_N_SHARDS, WD_OPT_RANK, WD_OPT_LOCAL_SHARDS, WD_OPT_LAUNCHES = 100, 101, 102, 103
 WD_OPT_GROUP_SIZE_USED = 104
+WD_OPT_REGION_ALIGN = 105
 WD_RANK_HANDLE_BYTES = 128
 # int (*)(uint64_t* value, int op, void* ctx)
 ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.POINTER(C.c_uint64), C.c_int, C.c_void_p)

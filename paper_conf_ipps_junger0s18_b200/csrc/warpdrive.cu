@@ -118,6 +118,7 @@ struct wd_table {
   int rank = 0;       // rank mode: this process's shard id
   int G = 4;          // |g|, or 0 = dynamic by load
   int G_used = 4;     // |g| of the current / last call
+  uint32_t align = 4; // A of reading C2': 16 for tables created with |g| >= 16, else 4
   uint64_t est_size = 0;   // host-side upper estimate of the stored keys (no sync needed)
   int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit
   int kif = 0;        // keys in flight per group (0 = default)
@@ -191,7 +192,7 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
   // C4': default p_max = nb — eq. 3 then visits every region, so an insert fails only when
   // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
-  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags, s.hseed};
+  const wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags, s.hseed, t->align};
   int grid = 1, block = 32;
   if (!t->serial) {
     block = wd::kBlock;
@@ -231,16 +232,19 @@ wd_status_t launch_gv(wd_table* t, Shard& s, const In& in, const Out& out, uint6
 // from measurements on B200 (tools/kbench.py split, profiles/r01_split.txt):
 //  * shard in half the L2 (<= 64 MB): one lane per window, K = 2 for 32/64-byte windows —
 //    instruction-lean (e.g. |g| = 8: 18 G inserts/s, 32 G queries/s at 2^22 keys);
-//  * from HBM: two lanes per window (V = min(|g|/2, 4)), K = 4 — a warp step then waits for
+//  * from HBM: two lanes per window (V = |g|/2), K = 2-4 — a warp step then waits for
 //    the slowest of 16 loads, not 32, with half the instructions of V = 1
 //    (|g| = 8, alpha 0.95, 2^28: 12.9 G inserts/s, 23.4 G queries/s vs 9.8 / 12.1 at V = 1).
-int choose_v(const wd_table* t, const Shard& s, int G) {
+//    Lanes load at most 32 B for inserts (V <= 4) and 64 B for queries (V <= 8):
+//    |g| = 16 queries 24.3 G/s at V = 8 vs 18.6 at V = 4, inserts 12.9 vs 13.5
+//    (tools/kbench.py cfg, profiles/r01_query_order.md).
+int choose_v(const wd_table* t, const Shard& s, int G, bool insert) {
   int v = t->spl;
   if (v == 0) {
     const bool small = s.cap * sizeof(unsigned long long) <= (64ull << 20);
     if (t->probe_mode == 1) v = 1;
     else if (t->probe_mode == 2 || small) v = G;
-    else v = G >= 2 ? std::max(1, std::min(G / 2, 4)) : 1;
+    else v = G >= 2 ? std::max(1, std::min(G / 2, insert ? 4 : 8)) : 1;
     if (G == 2 && t->probe_mode == 0) v = 2;
   }
   v = std::min(v, std::min(G, 8));
@@ -262,7 +266,7 @@ int choose_k(const wd_table* t, const Shard& s, int G, int V, bool insert) {
 template <int G, bool INSERT, class In, class Out>
 wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
-  const int v = choose_v(t, s, G), k = choose_k(t, s, G, v, INSERT);
+  const int v = choose_v(t, s, G, INSERT), k = choose_k(t, s, G, v, INSERT);
   if constexpr (G >= 8)
     if (v == 8) return launch_gv<G, 8, INSERT>(t, s, in, out, n_hint, st, k);
   if constexpr (G >= 4)
@@ -305,7 +309,7 @@ wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
   s.device = device;
   if (cap == 0) return fail(WD_ERR_INVALID_ARG, "capacity per shard exceeds 4 * 2^32 slots");
   s.cap = cap;
-  s.nb = (cap - 32) / wd::kRegionAlign + 1;
+  s.nb = (cap - 32) / t->align + 1;
   CK(cudaMalloc(&s.slots, cap * sizeof(unsigned long long)));
   CK(cudaMalloc(&s.counters, wd::CNT_N * sizeof(unsigned long long)));
   if (shared_main) {
@@ -872,13 +876,14 @@ wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* val
   }
   // P:245 future work, built: "a heuristic which dynamically scales the group size |g|
   // with the current load factor".  P:89 makes switching |g| between calls safe (same probe
-  // sequence).  Measured on B200 (profiles/r01_sweep.jsonl, 2^28 keys): |g| = 8 is fastest
-  // up to alpha ~0.95, |g| = 16 at 0.99.  The load used is the projected one after this call,
-  // from a host-side upper estimate of the size (no synchronisation).
+  // sequence).  Measured on B200 (profiles/r01_sweep.jsonl, 2^28 keys, insert + retrieve
+  // step): |g| = 8 is fastest up to alpha 0.9, |g| = 16 from 0.95 on (and for misses at any
+  // load).  The load used is the projected one after this call, from a host-side upper
+  // estimate of the size (no synchronisation).
   if (t->G == 0) {
     const double cap = double(wd_capacity(t));
     const double est = double(t->est_size) + (op == OP_INSERT ? double(n) : 0.0);
-    t->G_used = (est / cap > 0.97) ? 16 : 8;
+    t->G_used = (est / cap > 0.93) ? 16 : 8;
   }
   if (op == OP_INSERT) t->est_size = std::min<uint64_t>(t->est_size + n, wd_capacity(t));
   if (t->m == 1) {
@@ -906,6 +911,7 @@ wd_table* create_common(uint64_t capacity, int mode, int m, int group_size) {
   t->m = m;
   t->G = group_size;
   t->G_used = group_size ? group_size : 8;
+  t->align = wd::region_align_for(group_size);   // reading C2': fixed for the table's life
   return t;
 }
 
@@ -917,11 +923,10 @@ bool is_prime(uint64_t x) {
   return true;
 }
 
-// Reading C13': ceil(c/m) slots, rounded up to a multiple of A (C2) and
+// Reading C13': ceil(c/m) slots, rounded up to a multiple of A (C2') and
 // >= 32, then up until the number of region starts nb = (c-32)/A + 1 is prime, so eq. 3's
 // double hashing visits every region before repeating.  0 if nb would not fit 32 bits.
-uint64_t shard_cap(uint64_t capacity, int m) {
-  constexpr uint64_t A = wd::kRegionAlign;
+uint64_t shard_cap(uint64_t capacity, int m, uint64_t A) {
   uint64_t c = (capacity + m - 1) / m;
   c = round_up(std::max<uint64_t>(c, 32), A);
   uint64_t nb = (c - 32) / A + 1;
@@ -971,7 +976,7 @@ wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size) {
   int cur = 0;
   cudaGetDevice(&cur);
   cudaDeviceGetAttribute(&t->sm_count, cudaDevAttrMultiProcessorCount, n_gpus == 1 ? cur : 0);
-  const uint64_t c = shard_cap(capacity, n_gpus);
+  const uint64_t c = shard_cap(capacity, n_gpus, t->align);
   t->local.resize(n_gpus);
   for (int d = 0; d < n_gpus; ++d) {
     const int dev = n_gpus == 1 ? cur : d;
@@ -1008,7 +1013,7 @@ wd_table_t* wd_create_loopback(uint64_t capacity, int n_shards, int group_size) 
     delete t;
     return nullptr;
   }
-  const uint64_t c = shard_cap(capacity, n_shards);
+  const uint64_t c = shard_cap(capacity, n_shards, t->align);
   t->local.resize(n_shards);
   for (int d = 0; d < n_shards; ++d)
     if (shard_init(t, t->local[d], d, cur, c, t->loop_stream) != WD_OK) {
@@ -1035,7 +1040,7 @@ wd_table_t* wd_create_rank(uint64_t capacity, int rank, int world, int group_siz
   }
   cudaDeviceGetAttribute(&t->sm_count, cudaDevAttrMultiProcessorCount, cur);
   t->local.resize(1);
-  if (shard_init(t, t->local[0], rank, cur, shard_cap(capacity, world), nullptr) != WD_OK) {
+  if (shard_init(t, t->local[0], rank, cur, shard_cap(capacity, world, t->align), nullptr) != WD_OK) {
     wd_destroy(t);
     return nullptr;
   }
@@ -1269,6 +1274,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
   switch (opt) {
     case WD_OPT_GROUP_SIZE: return t->G;
     case WD_OPT_GROUP_SIZE_USED: return t->G_used;
+    case WD_OPT_REGION_ALIGN: return t->align;
     case WD_OPT_P_MAX: return t->pmax;
     case WD_OPT_BATCH: return int64_t(t->batch);
     case WD_OPT_SERIAL: return t->serial;

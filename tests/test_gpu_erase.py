@@ -62,15 +62,16 @@ def test_erase_and_reinsert_parity(wd, G, V):
     assert np.array_equal(gf, ef) and np.array_equal(gv, ev)
 
 
-@pytest.mark.parametrize("G,V", [(4, 1), (8, 4), (2, 2)])
+@pytest.mark.parametrize("G,V", [(4, 1), (8, 4), (2, 2), (16, 8), (16, 4)])
 def test_erase_rebuild_serial_layout(wd, G, V):
     # serial mode: insert, erase, rebuild — the slot words (incl. tombstones) equal the
     # oracle's sequential replay bit for bit at every stage
     n = 3000
-    c = oracle.physical_capacity(4000)
+    A = oracle.region_align_for(G)
+    c = oracle.physical_capacity(4000, A)
     keys, vals = wdgen.unique_keys(n, 91), wdgen.values(n, 92)
     er = keys[1::2]
-    r = oracle.Replay(c, G, p_max=oracle.n_regions(c))
+    r = oracle.Replay(c, G, p_max=oracle.n_regions(c, A), align=A)
     r.insert(keys, vals)
     r.erase(er)
     with wd.Table(4000, 1, G) as t:

@@ -43,7 +43,9 @@ def test_config1_unique_parity(wd, G, mode):
         assert t.size() == n
         cnt = t.counters()
         assert cnt["failed"] == 0 and cnt["reserved"] == 0
-        assert t.capacity() == oracle.physical_capacity(capacity_for(n, 0.95))
+        assert t.capacity() == oracle.physical_capacity(capacity_for(n, 0.95),
+                                                        oracle.region_align_for(G))
+        assert t.get_option(wd.WD_OPT_REGION_ALIGN) == oracle.region_align_for(G)
         load = t.size() / t.capacity()
         assert abs(load - 0.95) < 1e-3
     m, ev, ef = _oracle_answers(keys, vals, q)
@@ -76,10 +78,11 @@ def test_serial_layout_equals_fig3_replay(wd, G, mode):
     # the oracle's sequential replay of Fig. 3 bit for bit (probe sequence, windows,
     # leftmost-empty leader, update-on-match).
     n = 3000
-    c = oracle.physical_capacity(3200)
+    A = oracle.region_align_for(G)                  # reading C2': the table's geometry
+    c = oracle.physical_capacity(3200, A)
     keys = np.concatenate([wdgen.unique_keys(n, 3), wdgen.unique_keys(200, 3)])  # 200 updates
     vals = wdgen.values(n + 200, 4)
-    r = oracle.Replay(c, G)
+    r = oracle.Replay(c, G, align=A)
     r.insert(keys, vals)
     with wd.Table(3200, 1, G) as t:
         assert t.shard_capacity() == c
@@ -90,6 +93,33 @@ def test_serial_layout_equals_fig3_replay(wd, G, mode):
         slots = t.dump()
         assert t.size() == n
     assert np.array_equal(slots, r.table)
+
+
+@pytest.mark.parametrize("Gc,Gi", [(16, 4), (16, 1), (32, 8), (4, 16), (0, 16)])
+def test_region_align_is_per_table(wd, Gc, Gi):
+    # reading C2': A is fixed when the table is created (16 for |g| >= 16, else 4); later
+    # calls with another |g| probe the same sequence: the serial layout of a |g| = Gi
+    # insert equals the replay with the CREATION geometry, and queries with every |g| agree
+    n = 2000
+    A = oracle.region_align_for(Gc)
+    c = oracle.physical_capacity(2300, A)
+    keys, vals = wdgen.unique_keys(n, 51), wdgen.values(n, 52)
+    r = oracle.Replay(c, Gi, align=A)
+    r.insert(keys, vals)
+    with wd.Table(2300, 1, Gc) as t:
+        assert t.get_option(wd.WD_OPT_REGION_ALIGN) == A and t.capacity() == c
+        t.set_option(wd.WD_OPT_GROUP_SIZE, Gi)
+        t.set_option(wd.WD_OPT_SERIAL, 1)
+        t.insert(to_dev(keys), to_dev(vals))
+        assert t.sync() == 0
+        assert np.array_equal(t.dump(), r.table)
+        t.set_option(wd.WD_OPT_SERIAL, 0)
+        q = wdgen.interleaved_queries(n, 51)
+        cv, cf = oracle.expected_unique(q, n, 51, 52)
+        for Gq in (1, 4, 16, 32):
+            t.set_option(wd.WD_OPT_GROUP_SIZE, Gq)
+            ov, of = t.retrieve(to_dev(q))
+            assert np.array_equal(of.cpu().numpy(), cf) and np.array_equal(from_dev(ov), cv)
 
 
 @pytest.mark.parametrize("Gi,Gq,mi,mq", [(1, 32, 1, 1), (32, 1, 1, 2), (4, 8, 2, 1),
@@ -270,10 +300,11 @@ SPLITS = [(2, 2), (4, 2), (8, 2), (8, 4), (16, 4), (32, 8), (16, 2), (32, 4)]   
 def test_window_split_serial_layout(wd, G, V):
     # a window read by |g|/V lanes of V slots each: same probing, same sequential layout
     n = 2500
-    c = oracle.physical_capacity(2700)
+    A = oracle.region_align_for(G)
+    c = oracle.physical_capacity(2700, A)
     keys = np.concatenate([wdgen.unique_keys(n, 31), wdgen.unique_keys(100, 31)])
     vals = wdgen.values(n + 100, 32)
-    r = oracle.Replay(c, G)
+    r = oracle.Replay(c, G, align=A)
     r.insert(keys, vals)
     with wd.Table(2700, 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
