@@ -329,9 +329,11 @@ def main():
     roofline["other"] = roof(other)
     traffic_file = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(traffic_file) and world == 1:
-        tr = json.load(open(traffic_file)).get(f"{dom}_G{G}_a{args.alpha}_n{args.n_log2}")
-        if tr:
-            roofline["traffic"] = tr
+        tj = json.load(open(traffic_file))
+        for r, name in ((roofline, dom), (roofline["other"], other)):
+            tr = tj.get(f"{name}_G{G}_a{args.alpha}_n{args.n_log2}")
+            if tr:
+                r["traffic"] = tr
 
     # ---- e2e: the same step through the C-ABI with pinned host buffers
     e2e = None
