@@ -433,10 +433,45 @@ def run_sweep(args, wd, gg, torch):
                             "insert_gops": n / ims / 1e6, "query_gops": n / qms / 1e6,
                             "insert_frac": n * (40 + 32 * pc["ins_sectors"]) / (ims * 1e-3) / 1e9 / hbm,
                             "query_frac": n * (9 + 32 * pc["hit_sectors"]) / (qms * 1e-3) / 1e9 / hbm})
+    out += run_config1(wd, gg, torch)
     out += run_mix(wd, gg, torch, keys, vals, args.n_log2)
     del keys, vals, vout, fout
     out += run_zipf(wd, gg, torch)
     out += run_ooc(wd, gg, torch)
+    return out
+
+
+def run_config1(wd, gg, torch):
+    """BASELINE config 1: 2^20 unique pairs at alpha 0.95 (an 8.8 MB, L2-resident table),
+    then all 2^20 keys + 2^20 absent keys queried (interleaved); |g| = 4 as configured,
+    and 8 / 16 beside it.  Rates are per call (one launch each), device-resident."""
+    out = []
+    n = 1 << 20
+    keys, vals = gg.unique_keys(n, KEY_SEED), gg.values(n, VAL_SEED)
+    q = gg.interleaved_queries(n, KEY_SEED)
+    vout = torch.empty(2 * n, dtype=torch.int32, device="cuda")
+    fout = torch.empty(2 * n, dtype=torch.uint8, device="cuda")
+    s = torch.cuda.current_stream()
+    for G in (4, 8, 16):
+        with wd.Table(int(math.ceil(n / 0.95)), 1, G) as t:
+            ti, tq = [], []
+            for it in range(11):
+                a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+                t.clear(s)
+                a.record(s)
+                t.insert(keys, vals, s)
+                b.record(s)
+                t.retrieve(q, vout, fout, s)
+                c.record(s)
+                torch.cuda.synchronize()
+                if it:
+                    ti.append(a.elapsed_time(b))
+                    tq.append(b.elapsed_time(c))
+            assert t.sync() == 0 and t.size() == n and int(fout.sum().item()) == n
+            out.append({"sweep": "config1", "alpha": 0.95, "G": G, "keys": n, "queries": 2 * n,
+                        "table_MB": t.capacity() * 8 / 1e6,
+                        "insert_gops": n / (sum(ti) / len(ti)) / 1e6,
+                        "query_gops": 2 * n / (sum(tq) / len(tq)) / 1e6})
     return out
 
 
