@@ -38,8 +38,9 @@ def run(n, m, batch, reps=3, G=4):
 
 if __name__ == "__main__":
     lg = int(sys.argv[1]) if len(sys.argv) > 1 else 26
+    G = int(sys.argv[2]) if len(sys.argv) > 2 else 16
     n = 1 << lg
     for m in (1, 2, 4, 8):
-        i, q, l = run(n, m, 1 << 24)
-        print(f"n=2^{lg} loopback m={m} batch=2^24: insert {i:6.2f} G/s  query {q:6.2f} G/s  "
+        i, q, l = run(n, m, 1 << 24, G=G)
+        print(f"n=2^{lg} |g|={G} loopback m={m} batch=2^24: insert {i:6.2f} G/s  query {q:6.2f} G/s  "
               f"(launches {l})", flush=True)
