@@ -153,6 +153,53 @@ def cpu_baseline_sample(log2n: int = 26):
             "seconds": t2 - t0, "host_cpus": os.cpu_count()}
 
 
+def pcie_roofline(torch, n, te_ms, hk, hv, dk, dv, barrier):
+    """The e2e step's PCIe bound, measured live on this GPU with plain pinned copies of the
+    same buffers (cudaMemcpyAsync through torch): the insert must bring 8 B per pair
+    host -> device; the retrieve 4 B per key in while 5 B per result go out (concurrent, on
+    two streams).  bound = 8n / BW_h2d + max(4n / BW_h2d', 5n / BW_d2h'), primes = both
+    directions busy at once.  frac = bound / measured e2e step (1.0 = PCIe-limited)."""
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    ho = torch.empty(n, dtype=torch.int32, pin_memory=True)
+
+    def timed(fn, reps=3):
+        ts = []
+        for _ in range(reps + 1):
+            barrier()
+            t0 = time.perf_counter()
+            fn()
+            barrier()
+            ts.append(time.perf_counter() - t0)
+        return min(ts[1:])
+
+    def h2d():
+        with torch.cuda.stream(s1):
+            dk.copy_(hk, non_blocking=True)
+            dv.copy_(hv, non_blocking=True)
+
+    def both():
+        with torch.cuda.stream(s1):
+            dk.copy_(hk, non_blocking=True)
+        with torch.cuda.stream(s2):
+            ho.copy_(dv, non_blocking=True)
+
+    def d2h():
+        with torch.cuda.stream(s2):
+            ho.copy_(dv, non_blocking=True)
+
+    t_h2d = timed(h2d)                     # 8n bytes in
+    t_d2h = timed(d2h)                     # 4n bytes out
+    t_bi = timed(both)                     # 4n in || 4n out
+    bw_h2d = 8 * n / t_h2d / 1e9
+    bw_d2h = 4 * n / t_d2h / 1e9
+    bw_bi = 4 * n / t_bi / 1e9             # per direction with both busy
+    bound_ms = (8 * n / (bw_h2d * 1e9) + max(4 * n, 5 * n) / (bw_bi * 1e9)) * 1e3
+    del ho
+    return {"h2d_GBps": bw_h2d, "d2h_GBps": bw_d2h, "bidir_GBps_per_direction": bw_bi,
+            "bound_ms": bound_ms, "frac": bound_ms / te_ms,
+            "model": "8n/BW_h2d + 5n/BW_bidir (pinned cudaMemcpyAsync of the same buffers)"}
+
+
 def workload_config(args, world):
     n = 1 << args.n_log2
     return {"workload": f"config2: 2^{args.n_log2} unique u32 key/value pairs per GPU, "
@@ -323,7 +370,28 @@ def main():
                 "sectors_per_op": pc["ins_sectors" if name == "insert" else "hit_sectors"],
                 # HBM moves whole 128-B lines for random accesses (C2): the
                 # same kernel against the replay's distinct lines per op
-                "line_model": line_model(name, ms)}
+                "line_model": line_model(name, ms),
+                # the same kernel against the MEASURED random-access rate of its own access
+                # pattern on this part (tools/randbench.cu -> profiles/ceilings.json)
+                "pattern_ceiling": pattern_ceiling(name, ms)}
+
+    def pattern_ceiling(name, ms):
+        cf = os.path.join(ROOT, "profiles", "ceilings.json")
+        if not os.path.exists(cf):
+            return None
+        c = json.load(open(cf))
+        wb = str(8 * G)
+        L = pc["ins_windows" if name == "insert" else "hit_windows"]
+        R = c["read"].get(wb)
+        C = c["casw"].get(wb)
+        if R is None or (name == "insert" and C is None):
+            return None
+        t = (L - 1) / R + 1 / C if name == "insert" else L / R      # ns per op
+        ach = n / (ms * 1e-3) / 1e9
+        return {"gops": 1 / t, "achieved_gops": ach, "frac": ach * t, "windows_per_op": L,
+                "model": ("(L-1) random %s-B window reads + 1 read-then-CAS (randbench casw)"
+                          if name == "insert" else "L random %s-B window reads") % wb,
+                "rates_Gwin_s": {"read": R, "casw": C}, "source": "profiles/ceilings.json"}
 
     def line_model(name, ms):
         lines = pc.get("ins_lines" if name == "insert" else "hit_lines")
@@ -375,6 +443,9 @@ def main():
         e2e = {"value": ops / (te * 1e-3) / 1e9, "unit": UNIT, "ms_per_step": te,
                "h2d_bytes_per_step": 12 * n, "d2h_bytes_per_step": 5 * n, "steps": e_steps}
         assert table.sync() == 0
+        del hvo, hfo
+        e2e["pcie"] = pcie_roofline(torch, n, te, hk, hv, keys, vals, barrier)
+        del hk, hv
 
     # ---- CPU baseline (rank 0, N = 1 only)
     cpu = None

@@ -204,6 +204,8 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
     const uint64_t keys_per_block = uint64_t(wd::kBlock / 32) * K * (32 / (G / V));
     const uint64_t need = std::max<uint64_t>(1, (n_hint + keys_per_block - 1) / keys_per_block);
     grid = static_cast<int>(std::min<uint64_t>(need, uint64_t(t->sm_count) * blocks_per_sm(kern)));
+    static const int cap_env = getenv("WD_MAX_BLOCKS") ? atoi(getenv("WD_MAX_BLOCKS")) : 0;
+    if (cap_env > 0) grid = std::min(grid, cap_env);   // measurement hook (tools/)
   }
   kern<<<grid, block, 0, st>>>(tv, in, out, s.counters, t->serial);
   CK(cudaGetLastError());

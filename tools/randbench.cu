@@ -211,6 +211,8 @@ int main() {
     run<8, 2, 32, 32>("casw", buf, bytes, grid, it, sink);
     run<8, 1, 64, 64>("cas", buf, bytes, grid, it, sink);
     run<8, 2, 64, 64>("casw", buf, bytes, grid, it, sink);
+    run<8, 1, 128, 128>("cas", buf, bytes, grid, it, sink);
+    run<8, 2, 128, 128>("casw", buf, bytes, grid, it, sink);
     {
       const int grid = sms * 4, kpc = 32;
       const size_t nk = size_t(grid) * 256 * 8 * kpc;
