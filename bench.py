@@ -79,7 +79,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
-                 "--format=csv,noheader,nounits", "-lms", "200"],
+                 "--format=csv,noheader,nounits", "-lms", "50"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.th = threading.Thread(target=self._read, daemon=True)
             self.th.start()
@@ -267,10 +267,12 @@ def main():
     dev = 0 if args.same_device else local_rank
     torch.cuda.set_device(dev)
     if world > 1:
-        if args.dist_backend == "nccl":
+        # NCCL refuses two ranks on one device: the same-device dry run uses gloo
+        backend = "gloo" if args.same_device else args.dist_backend
+        if backend == "nccl":
             dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
         else:
-            dist.init_process_group(args.dist_backend)
+            dist.init_process_group(backend)
 
     n = 1 << args.n_log2
     G = args.group_size
