@@ -9,8 +9,9 @@
 //                     on three streams with double-buffered staging (Fig. 5).
 //   cascade (m > 1) . per batch: multisplit fused with the push into the owners'
 //                     receive regions -> publish T row + ready flags -> owner waits for its
-//                     T column -> local insert / query -> done flags -> (query) origin
-//                     pulls results back and unpermutes -> consumed flags.  All signalling
+//                     T column -> local insert / query, results pushed back into the
+//                     origins' result regions -> done flags -> (query) origin unpermutes
+//                     from its own memory -> consumed flags.  All signalling
 //                     is device-side (no host synchronisation per batch); receive and
 //                     result regions are double-buffered by epoch parity.
 // =====================================================================================
@@ -76,7 +77,7 @@ struct DeviceGuard {
 // pointers into one shard's exchange arena, valid in this process (own or peer-mapped)
 struct PeerView {
   unsigned long long* recv[2] = {nullptr, nullptr};        // [m][B] items written by senders
-  unsigned long long* res[2] = {nullptr, nullptr};         // [m][B] packed query results
+  unsigned long long* res[2] = {nullptr, nullptr};         // [m][B] packed query results, region d pushed by owner d
   unsigned long long* recv_count[2] = {nullptr, nullptr};  // [m] column of T
   unsigned long long* flags = nullptr;                     // [FLAG_N][m]
 };
@@ -473,13 +474,22 @@ wd_status_t exchange_init_shard(wd_table* t, Shard& s, uint64_t B) {
 
 wd_status_t rank_allgather_views(wd_table* t, uint64_t B);
 
+// Items per shard per cascade batch: WD_OPT_BATCH rounded up to a power of two, so the
+// exchange regions sit a power of two apart and the owner's result push (OutPacked) finds
+// its target region with a shift.
+uint64_t xchg_batch(const wd_table* t) {
+  uint64_t b = 1;
+  while (b < t->batch) b <<= 1;
+  return b;
+}
+
 // (re)build the exchange arenas for batch size B (collective in rank mode)
 wd_status_t ensure_exchange(wd_table* t) {
   if (t->m == 1) return WD_OK;
-  if (t->xbatch == t->batch) return WD_OK;
+  if (t->xbatch == xchg_batch(t)) return WD_OK;
   if (t->mode == MODE_RANK && t->connected)
     return fail(WD_ERR_INVALID_ARG, "rank mode: batch size fixed after wd_rank_connect");
-  const uint64_t B = t->batch;
+  const uint64_t B = xchg_batch(t);
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
     CK(cudaStreamSynchronize(s.s_main));
@@ -705,7 +715,7 @@ wd_status_t agree_batches(wd_table* t, uint64_t local_nbt, uint64_t* global_nbt)
 wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t stream) {
   const bool insert = op == OP_INSERT;
   TRY(ensure_exchange(t));
-  const uint64_t B = t->batch;
+  const uint64_t B = t->xbatch;   // a power of two (xchg_batch)
   const int m = t->m;
   uint64_t local_nbt = 0;
   for (size_t r = 0; r < t->local.size(); ++r) {
@@ -726,9 +736,10 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
   //   A (s_main):  multisplit fused with the push into the owners' receive regions, then
   //                publish the row of T and the READY flags
   //   B (s_probe): wait for the column of T, probe (insert / retrieve), DONE flags
-  //   C (s_main):  queries only — pull the results back, unpermute, RESC flags
+  //   C (s_main):  queries only — unpermute the results the owners pushed into this shard's
+  //                result slot (local gather), RESC flags (the slot may be reused)
   // Issued as A(0), then A(b+1), B(b), C(b): the multisplit and transposition of batch b+1
-  // overlap the probing of batch b (Fig. 5's MST || INS), and the query's reverse pull of
+  // overlap the probing of batch b (Fig. 5's MST || INS), and the query's unpermute of
   // batch b never blocks the next multisplit.  Cross-shard ordering is by epoch flags only.
   const unsigned long long e0 = t->epoch;
   auto phaseA = [&](uint64_t b) -> wd_status_t {
@@ -786,10 +797,16 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
         // origins consumed the results of the previous query epoch that used this slot
         if (t->res_used[slot]) TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
         const wd::InSeg<false> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
+        // reverse transposition: results go straight to their origins' result
+        // slots (region s.id of origin d's slot), coalesced remote stores
+        wd::OutPacked out{};
+        out.stride = B;
+        out.shift = __builtin_ctzll(B);
+        for (int d = 0; d < m; ++d) out.seg[d] = t->peers[d].res[slot] + uint64_t(s.id) * B;
         if (op == OP_ERASE)
-          TRY(launch_probe<false>(t, s, in, wd::OutErase<wd::OutPacked>{{s.self.res[slot]}}, B, s.s_probe));
+          TRY(launch_probe<false>(t, s, in, wd::OutErase<wd::OutPacked>{out}, B, s.s_probe));
         else
-          TRY(launch_probe<false>(t, s, in, wd::OutPacked{s.self.res[slot]}, B, s.s_probe));
+          TRY(launch_probe<false>(t, s, in, out, B, s.s_probe));
       }
       TRY(launch_signal(t, s, s.s_probe, FLAG_DONE, e));
     }
@@ -807,7 +824,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e));
       if (cnt) {
         wd::DstPtrs src{};
-        for (int d = 0; d < m; ++d) src.p[d] = t->peers[d].res[slot] + uint64_t(s.id) * B;
+        for (int d = 0; d < m; ++d) src.p[d] = s.self.res[slot] + uint64_t(d) * B;   // local
         uint32_t* ov; uint8_t* of;
         out_ptrs(s, io, off, int(b % kStage), &ov, &of);
         const int grid = int(std::min<uint64_t>((cnt + wd::kBlock - 1) / wd::kBlock,
