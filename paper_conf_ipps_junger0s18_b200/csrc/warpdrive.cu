@@ -760,7 +760,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
           else dst.p[d] = reinterpret_cast<uint32_t*>(t->peers[d].recv[slot]) + uint64_t(s.id) * B;
         }
         // every resident block of the SM (occupancy API): more tiles in flight per SM
-        const uint64_t tiles = (cnt + wd::kBlock * 8 - 1) / (wd::kBlock * 8);
+        const uint64_t tiles = (cnt + wd::kMsTile - 1) / wd::kMsTile;
         const int per_sm = insert ? blocks_per_sm(wd::multisplit_kernel<true>)
                                   : blocks_per_sm(wd::multisplit_kernel<false>);
         const int grid = int(std::min<uint64_t>(tiles, uint64_t(t->sm_count) * per_sm));
