@@ -226,13 +226,15 @@ def test_edge_cases(wd):
 
 
 @pytest.mark.parametrize("pinned", [True, False])
-def test_host_pointers_out_of_core(wd, pinned):
-    # a11: host-resident input streamed in batches; tiny batch -> many batches
+@pytest.mark.parametrize("batch", [7_777, 25_001, 1 << 20])
+def test_host_pointers_out_of_core(wd, pinned, batch):
+    # a11: host-resident input streamed in batches.  7 777: many batches (the
+    # staging slots are reused); 25 001: full batches + a ragged last one; 2^20: one batch
     n = 100_003
     keys, vals = wdgen.unique_keys(n, 13), wdgen.values(n, 14)
     q = wdgen.interleaved_queries(n, 13)
     with wd.Table(capacity_for(n, 0.95), 1, 4) as t:
-        t.set_option(wd.WD_OPT_BATCH, 7_777)
+        t.set_option(wd.WD_OPT_BATCH, batch)
         if pinned:
             gv, gf = gpu_roundtrip(t, keys, vals, q, host=True)
         else:
