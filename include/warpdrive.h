@@ -176,6 +176,12 @@ typedef enum {
                                 vector load, so a window is read by |g|/V lanes (1: the
                                 paper's cooperative group; |g|: one lane).  0 = from
                                 WD_OPT_PROBE_MODE.  V in {1,2,4,8}, V <= |g|. */
+    WD_OPT_SPAN = 10,        /* S: windows one lane loads per round trip in the one-lane-per-
+                                window mode (V = |g| <= 4, single-shard calls): the lane decides
+                                on the first of the S windows holding a match or an empty slot
+                                (Fig. 3 order), so results and layout do not depend on S.
+                                0 (default): 2 for tables of <= 64 MB and for |g| = 1, else 1;
+                                1: off; 2: on. */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -22,6 +22,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <type_traits>
 #include <unordered_map>
 #include <vector>
 
@@ -130,6 +131,7 @@ struct wd_table {
   int kif = 0;        // keys in flight per group (0 = default)
   int probe_mode = 0; // 0: auto, 1: cooperative groups (Fig. 3), 2: lane-window (|g| <= 8)
   int spl = 0;        // slots per lane V (WD_OPT_SLOTS_PER_LANE; 0 = from probe mode)
+  int span = 0;       // windows per lane load S (WD_OPT_SPAN; 0 = auto)
   // wd::kF_* kernel variants (WD_OPT_KERNEL_FLAGS).  Default all three: atom.exch value
   // updates take hot (Zipf) keys from 0.5 to 6-8 G inserts/s (tools/flags_bench.py),
   // L1-allowed probe loads add ~15 % there; the scrambled query chunk order adds 22-40 % to
@@ -191,10 +193,10 @@ int blocks_per_sm(K kern) {
 }
 
 // ------------------------------------------------------------------ probe dispatch
-template <int G, int V, int K, bool INSERT, class In, class Out>
+template <int G, int V, int K, bool INSERT, class In, class Out, int S = 1>
 wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
-  auto kern = wd::probe_kernel<G, V, K, INSERT, In, Out>;
+  auto kern = wd::probe_kernel<G, V, K, INSERT, In, Out, S>;
   // C4': default p_max = nb — eq. 3 then visits every region, so an insert fails only when
   // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
@@ -216,9 +218,28 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
 
 // instantiated (|g|, V, K) combinations: V = slots per lane (1: the paper's cooperative
 // group of |g| lanes; |g|: one lane per window), K = keys in flight per group
+// windows per lane load S (span read-ahead, one lane per window): 2 for L2-resident tables
+// with |g| <= 4 — calls on them are bound by the longest probe chain, not by bandwidth
+// (profiles/r01_small_calls.md), and S = 2 halves its round trips — and for |g| = 1 at any
+// size (7 windows per insert at alpha 0.95).  Measured (tools/span_bench.py,
+// profiles/r01_span.txt): config 1 (2^20 keys, |g| = 4) 5.4 -> 9.1 G inserts/s and
+// 5.9 -> 8.8 G queries/s; |g| = 1 at 2^26 keys 3.9 -> 7.3 G inserts/s (queries equal).
+// Single-shard input only.
+int choose_span(const wd_table* t, const Shard& s, int G, int V) {
+  if (V != G || G > 4 || t->span == 1) return 1;
+  if (t->span == 2 || G == 1) return 2;
+  return s.cap * sizeof(unsigned long long) <= (64ull << 20) ? 2 : 1;
+}
+
 template <int G, int V, bool INSERT, class In, class Out>
 wd_status_t launch_gv(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                       cudaStream_t st, int k) {
+  if constexpr (V == G && G <= 4 && std::is_same_v<In, wd::InSoA>) {
+    // span read-ahead variants, at the K the auto choice uses for these (G, V)
+    constexpr int KS = G == 1 ? 8 : G == 2 ? 4 : 2;
+    if (k == KS && choose_span(t, s, G, V) == 2)
+      return launch_probe_k<G, V, KS, INSERT, In, Out, 2>(t, s, in, out, n_hint, st);
+  }
   if constexpr (V == 1) {
     if (k == 2) return launch_probe_k<G, 1, 2, INSERT>(t, s, in, out, n_hint, st);
     if (k == 4) return launch_probe_k<G, 1, 4, INSERT>(t, s, in, out, n_hint, st);
@@ -1293,6 +1314,10 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       if (v != 0 && v != 1) return fail(WD_ERR_INVALID_ARG, "partition mode %lld", (long long)v);
       t->pmode = int(v);
       return WD_OK;
+    case WD_OPT_SPAN:
+      if (v < 0 || v > 2) return fail(WD_ERR_INVALID_ARG, "span %lld", (long long)v);
+      t->span = int(v);
+      return WD_OK;
     default: return fail(WD_ERR_INVALID_ARG, "option %d is read-only or unknown", int(opt));
   }
 }
@@ -1312,6 +1337,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_KERNEL_FLAGS: return t->kflags;
     case WD_OPT_SLOTS_PER_LANE: return t->spl;
     case WD_OPT_PART_MODE: return t->pmode;
+    case WD_OPT_SPAN: return t->span;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;
     case WD_OPT_LOCAL_SHARDS: return int64_t(t->local.size());

@@ -405,3 +405,40 @@ def test_dynamic_group_size_by_load(wd):
         assert t.sync() == 0 and t.size() == n
     cv, cf = oracle.expected_unique(q, n, 121, 122)
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
+@pytest.mark.parametrize("G", [1, 2, 4])
+@pytest.mark.parametrize("span", [1, 2])
+def test_span_read_ahead(wd, G, span):
+    # WD_OPT_SPAN: one lane loads S = 2 consecutive windows per round trip and decides on
+    # the first that holds a match or an empty slot (Fig. 3 order).  The serial layout must
+    # still equal the sequential replay bit for bit, and concurrent calls must return the
+    # exact map — hits, misses (long chains at alpha 0.99) and updates.
+    n = 2500
+    A = oracle.region_align_for(G)
+    c = oracle.physical_capacity(2700, A)
+    keys = np.concatenate([wdgen.unique_keys(n, 51), wdgen.unique_keys(100, 51)])
+    vals = wdgen.values(n + 100, 52)
+    r = oracle.Replay(c, G, align=A)
+    r.insert(keys, vals)
+    with wd.Table(2700, 1, G) as t:
+        t.set_option(wd.WD_OPT_PROBE_MODE, 2)          # one lane per window (V = |g|)
+        t.set_option(wd.WD_OPT_SPAN, span)
+        assert t.get_option(wd.WD_OPT_SPAN) == span
+        t.set_option(wd.WD_OPT_SERIAL, 1)
+        t.insert(to_dev(keys), to_dev(vals))
+        assert t.sync() == 0
+        assert np.array_equal(t.dump(), r.table)
+    n = 99_001
+    keys, vals = wdgen.unique_keys(n, 53), wdgen.values(n, 54)
+    q = wdgen.interleaved_queries(n, 53)
+    with wd.Table(capacity_for(n, 0.99), 1, G) as t:
+        t.set_option(wd.WD_OPT_PROBE_MODE, 2)
+        t.set_option(wd.WD_OPT_SPAN, span)
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0 and t.size() == n
+        df = t.erase(to_dev(q[: n // 2]))             # deletion runs the same probe
+        assert t.sync() == 0
+    cv, cf = oracle.expected_unique(q, n, 53, 54)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+    assert np.array_equal(df.cpu().numpy().astype(bool), cf[: n // 2].astype(bool))
