@@ -154,8 +154,10 @@ typedef enum {
                                 load of 0.93 (measured on B200) */
     WD_OPT_P_MAX = 1,        /* outer probing bound p_max (Fig. 3 Line 4); 0 (default) = the
                                 number of regions nb, i.e. fail only when the table is full (C4') */
-    WD_OPT_BATCH = 2,        /* items per shard per pipeline batch (2^24); multi-shard
-                                calls round it up to a power of two */
+    WD_OPT_BATCH = 2,        /* items per shard per pipeline batch; multi-shard calls round it
+                                up to a power of two.  Default: 2^24 for the multi-shard
+                                cascade, 2^22 for single-shard host streaming (shorter
+                                pipeline fill/drain, measured) unless set explicitly */
     WD_OPT_SERIAL = 3,       /* 1: one probing group, one key at a time (deterministic
                                 layout, test hook for the Fig. 3 replay) */
     WD_OPT_KEYS_IN_FLIGHT = 4, /* 0 = default; else keys per group in flight (1,2,4,8) */

@@ -138,6 +138,7 @@ struct wd_table {
   // queries issued in insert order (profiles/r01_query_order.md).
   uint32_t kflags = wd::kF_L1 | wd::kF_XCHG | wd::kF_QSCR;
   uint64_t batch = 1ull << 24;
+  bool batch_set = false;  // WD_OPT_BATCH given: the single-shard pipeline uses it as is
   int serial = 0;
   uint32_t pseed = 0x9E3779B9u;
   int pmode = 0;
@@ -684,8 +685,11 @@ wd_status_t single_op(wd_table* t, int op, const IO& io, cudaStream_t stream) {
     const wd::InSoA in{io.keys, io.vals, io.n};
     return probe_soa(t, s, op, in, io.vout, io.fout, io.n, stream);
   }
-  // out-of-core pipeline (Fig. 5): H2D(b+1) || probe(b) || D2H(b-1)
-  const uint64_t B = t->batch;
+  // out-of-core pipeline (Fig. 5): H2D(b+1) || probe(b) || D2H(b-1).  Default
+  // batch here 2^22 (not P:197's 2^24): shorter pipeline fill and drain; the bench's e2e
+  // step (2^28 pairs, pinned) took 67.7 / 68.0 / 69.7 / 72.5 ms at 2^22 / 2^23 / 2^24 /
+  // 2^25 (tools/e2e_batch.py, profiles/r01_e2e_batch.txt)
+  const uint64_t B = t->batch_set ? t->batch : std::min<uint64_t>(t->batch, 1ull << 22);
   TRY(ensure_staging(s, B, io.kin == PK_PAGEABLE || io.kout == PK_PAGEABLE));
   cudaEvent_t ev0;
   TRY(fork_from(t, stream, &ev0));
@@ -1290,6 +1294,7 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
     case WD_OPT_BATCH:
       if (v < 1 || v > (1ll << wd::kPosShift)) return fail(WD_ERR_INVALID_ARG, "batch %lld", (long long)v);
       t->batch = uint64_t(v);
+      t->batch_set = true;
       return WD_OK;
     case WD_OPT_SERIAL: t->serial = v ? 1 : 0; return WD_OK;
     case WD_OPT_KEYS_IN_FLIGHT:
