@@ -61,6 +61,9 @@ def parse():
                     help="torch.distributed backend for the control plane (gloo: tests)")
     ap.add_argument("--same-device", action="store_true",
                     help="all ranks on cuda:0 (dry run of the N>1 path on a 1-GPU box)")
+    ap.add_argument("--strong", action="store_true",
+                    help="strong scaling (Fig. 9, eq. 4): 2^n-log2 pairs in total, split over "
+                         "the ranks (default: weak, 2^n-log2 pairs per GPU)")
     ap.add_argument("--sweep", action="store_true",
                     help="extra lines: config-2 alpha x |g| sweep (not the headline)")
     return ap.parse_args()
@@ -201,8 +204,9 @@ def pcie_roofline(torch, n, te_ms, hk, hv, dk, dv, barrier):
 
 
 def workload_config(args, world):
-    n = 1 << args.n_log2
-    return {"workload": f"config2: 2^{args.n_log2} unique u32 key/value pairs per GPU, "
+    n = (1 << args.n_log2) // (world if args.strong else 1)
+    per = "in total" if args.strong else "per GPU"
+    return {"workload": f"config2: 2^{args.n_log2} unique u32 key/value pairs {per}, "
                         f"load {args.alpha}, |g|={args.group_size}; step = fill + insert all + "
                         f"retrieve all (100% hits, queried in insert order)",
             "global_batch": n * world, "pairs_per_gpu": n, "alpha": args.alpha,
@@ -237,8 +241,8 @@ def run_reference(args):
     val = 2 * n / t / 1e9
     line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
-            "data": "synthetic", "impl": "reference",
+            "higher_is_better": True, "scaling": "strong" if args.strong else "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic", "impl": "reference",
             "config": dict(workload_config(args, args.gpus),
                            reference_sample="bounded 2^22 unique inserts + 2^22 hit queries "
                                             "per step, single-threaded C oracle"),
@@ -274,7 +278,8 @@ def main():
         else:
             dist.init_process_group(backend)
 
-    n = 1 << args.n_log2
+    # weak scaling: n pairs per GPU; strong (--strong): 2^n-log2 in total, n per GPU
+    n = (1 << args.n_log2) // (world if args.strong else 1)
     G = args.group_size
     cap_local = int(math.ceil(n / args.alpha))
     if world > 1:
@@ -461,8 +466,8 @@ def main():
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_ms,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-            "dtype": "u32", "data": "synthetic",
+            "higher_is_better": True, "scaling": "strong" if args.strong else "weak",
+            "vs_baseline": None, "dtype": "u32", "data": "synthetic",
             "config": dict(workload_config(args, world),
                            capacity_per_gpu=table.shard_capacity(0)),
             "insert_gops": n * world / (ins_ms * 1e-3) / 1e9,
