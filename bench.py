@@ -158,49 +158,53 @@ def cpu_baseline_sample(log2n: int = 26):
 
 def pcie_roofline(torch, n, te_ms, hk, hv, dk, dv, barrier):
     """The e2e step's PCIe bound, measured live on this GPU with plain pinned copies of the
-    same buffers (cudaMemcpyAsync through torch): the insert must bring 8 B per pair
-    host -> device; the retrieve 4 B per key in while 5 B per result go out (concurrent, on
-    two streams).  bound = 8n / BW_h2d + max(4n / BW_h2d', 5n / BW_d2h'), primes = both
-    directions busy at once.  frac = bound / measured e2e step (1.0 = PCIe-limited)."""
+    same buffers (cudaMemcpyAsync through torch): the insert must bring 8n bytes host ->
+    device (t_ins); the retrieve brings 4n bytes in while 5n bytes (values + found flags) go
+    out, both directions at once on two streams (t_ret).  bound = t_ins + t_ret, each the
+    best of 5 timed repetitions; frac = bound / measured e2e step (1.0 = PCIe-limited)."""
     s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
     ho = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    hf = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+    df = torch.empty(n, dtype=torch.uint8, device="cuda")
+    cur = torch.cuda.current_stream()
 
-    def timed(fn, reps=3):
+    def timed(fn, reps=5):
         ts = []
         for _ in range(reps + 1):
             barrier()
-            t0 = time.perf_counter()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(cur)
+            s1.wait_stream(cur)
+            s2.wait_stream(cur)
             fn()
+            cur.wait_stream(s1)
+            cur.wait_stream(s2)
+            b.record(cur)
             barrier()
-            ts.append(time.perf_counter() - t0)
+            ts.append(a.elapsed_time(b) * 1e-3)
         return min(ts[1:])
 
-    def h2d():
+    def ins():
         with torch.cuda.stream(s1):
             dk.copy_(hk, non_blocking=True)
             dv.copy_(hv, non_blocking=True)
 
-    def both():
+    def ret():
         with torch.cuda.stream(s1):
             dk.copy_(hk, non_blocking=True)
         with torch.cuda.stream(s2):
             ho.copy_(dv, non_blocking=True)
+            hf.copy_(df, non_blocking=True)
 
-    def d2h():
-        with torch.cuda.stream(s2):
-            ho.copy_(dv, non_blocking=True)
-
-    t_h2d = timed(h2d)                     # 8n bytes in
-    t_d2h = timed(d2h)                     # 4n bytes out
-    t_bi = timed(both)                     # 4n in || 4n out
-    bw_h2d = 8 * n / t_h2d / 1e9
-    bw_d2h = 4 * n / t_d2h / 1e9
-    bw_bi = 4 * n / t_bi / 1e9             # per direction with both busy
-    bound_ms = (8 * n / (bw_h2d * 1e9) + max(4 * n, 5 * n) / (bw_bi * 1e9)) * 1e3
-    del ho
-    return {"h2d_GBps": bw_h2d, "d2h_GBps": bw_d2h, "bidir_GBps_per_direction": bw_bi,
+    t_ins = timed(ins)                     # 8n bytes in
+    t_ret = timed(ret)                     # 4n in || 5n out
+    del ho, hf, df
+    bound_ms = (t_ins + t_ret) * 1e3
+    return {"h2d_GBps": 8 * n / t_ins / 1e9, "retrieve_in_out_GBps": 9 * n / t_ret / 1e9,
+            "insert_copy_ms": t_ins * 1e3, "retrieve_copy_ms": t_ret * 1e3,
             "bound_ms": bound_ms, "frac": bound_ms / te_ms,
-            "model": "8n/BW_h2d + 5n/BW_bidir (pinned cudaMemcpyAsync of the same buffers)"}
+            "model": "copy(8n in) + copy(4n in || 5n out), pinned cudaMemcpyAsync of the "
+                     "same buffers, CUDA events, best of 5"}
 
 
 def workload_config(args, world):

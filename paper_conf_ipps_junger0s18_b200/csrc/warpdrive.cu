@@ -265,16 +265,18 @@ wd_status_t launch_gv(wd_table* t, Shard& s, const In& in, const Out& out, uint6
 //  * from HBM: two lanes per window (V = |g|/2), K = 2-4 — a warp step then waits for
 //    the slowest of 16 loads, not 32, with half the instructions of V = 1
 //    (|g| = 8, alpha 0.95, 2^28: 12.9 G inserts/s, 23.4 G queries/s vs 9.8 / 12.1 at V = 1).
-//    Lanes load at most 32 B for inserts (V <= 4) and 64 B for queries (V <= 8):
-//    |g| = 16 queries 24.3 G/s at V = 8 vs 18.6 at V = 4, inserts 12.9 vs 13.5
-//    (tools/kbench.py cfg, profiles/r01_query_order.md).
+//    Lanes load at most 64 B (V <= 8), inserts on 32-B-aligned tables at most 32 B (V <= 4):
+//    |g| = 16 queries 24.3 G/s at V = 8 vs 18.6 at V = 4 (profiles/r01_query_order.md);
+//    on line-aligned tables (A = 16, reading C2') inserts too: |g| = 16 14.3 -> 15.0 G/s,
+//    |g| = 32 10.9 -> 12.9 G/s at V = 8, while |g| = 8 (A = 4) drops 12.9 -> 8.3
+//    (tools/kbench.py cfg, profiles/r01_ab_insert_v8.txt).
 int choose_v(const wd_table* t, const Shard& s, int G, bool insert) {
   int v = t->spl;
   if (v == 0) {
     const bool small = s.cap * sizeof(unsigned long long) <= (64ull << 20);
     if (t->probe_mode == 1) v = 1;
     else if (t->probe_mode == 2 || small) v = G;
-    else v = G >= 2 ? std::max(1, std::min(G / 2, insert ? 4 : 8)) : 1;
+    else v = G >= 2 ? std::max(1, std::min(G / 2, insert && t->align < 16 ? 4 : 8)) : 1;
     if (G == 2 && t->probe_mode == 0) v = 2;
   }
   v = std::min(v, std::min(G, 8));
