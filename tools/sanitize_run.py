@@ -11,7 +11,7 @@ q = wdgen.interleaved_queries(n, 1)
 cv, cf = oracle.expected_unique(q, n, 1, 2)
 def check(gv, gf):
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
-for G, V in [(4, 1), (8, 4), (4, 4), (1, 1), (32, 8)]:
+for G, V in [(4, 1), (8, 4), (4, 4), (1, 1), (2, 2), (16, 8), (32, 8)]:  # (1,1), (2,2), (4,4): span S = 2
     with wd.Table(capacity_for(n, 0.9), 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
         check(*gpu_roundtrip(t, keys, vals, q))
