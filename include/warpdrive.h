@@ -184,6 +184,13 @@ typedef enum {
                                 (Fig. 3 order), so results and layout do not depend on S.
                                 0 (default): 2 for tables of <= 64 MB and for |g| = 1, else 1;
                                 1: off; 2: on. */
+    WD_OPT_SLICES = 11,      /* a bulk insert of device-resident pairs into a single-shard table
+                                is grouped by table slice of the keys' first region (Line 5) and
+                                inserted with one probe launch per slice (better L2 reuse); the
+                                probing of each key is unchanged.  0 (default): 16 slices for
+                                tables > 512 MB and calls of >= 2^22 pairs, else 1 (off);
+                                1: off; 2..32: that many slices.  Uses 8 B of scratch per pair,
+                                at most 2^26 pairs at a time. */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -30,7 +30,7 @@ WD_NOT_FOUND = 0xFFFFFFFF
 
 WD_OPT_GROUP_SIZE, WD_OPT_P_MAX, WD_OPT_BATCH, WD_OPT_SERIAL = 0, 1, 2, 3
 WD_OPT_KEYS_IN_FLIGHT, WD_OPT_PART_SEED, WD_OPT_PART_MODE, WD_OPT_PROBE_MODE = 4, 5, 6, 7
-WD_OPT_KERNEL_FLAGS, WD_OPT_SLOTS_PER_LANE, WD_OPT_SPAN = 8, 9, 10
+WD_OPT_KERNEL_FLAGS, WD_OPT_SLOTS_PER_LANE, WD_OPT_SPAN, WD_OPT_SLICES = 8, 9, 10, 11
 WD_OPT_N_SHARDS, WD_OPT_RANK, WD_OPT_LOCAL_SHARDS, WD_OPT_LAUNCHES = 100, 101, 102, 103
 WD_OPT_GROUP_SIZE_USED = 104
 WD_OPT_REGION_ALIGN = 105

@@ -95,6 +95,13 @@ struct Shard {
   uint32_t hseed = 0;            // hash seed of the current table (changes on rebuild)
   unsigned long long* slots = nullptr;
   unsigned long long* counters = nullptr;
+  // slice-grouped bulk insert (slice_insert): packed-pair scratch for one chunk, and
+  // counts[32] | bounds[33] | cursor[32]; sl_done orders reuse across streams
+  unsigned long long* sl_buf = nullptr;
+  uint64_t sl_cap = 0;
+  unsigned long long* sl_meta = nullptr;
+  cudaEvent_t sl_done = nullptr;
+  bool sl_used = false;
   cudaStream_t s_main = nullptr, s_h2d = nullptr, s_d2h = nullptr;
   cudaStream_t s_probe = nullptr;   // phase B of the cascade (own stream unless loopback)
   bool own_main = true;
@@ -132,6 +139,7 @@ struct wd_table {
   int probe_mode = 0; // 0: auto, 1: cooperative groups (Fig. 3), 2: lane-window (|g| <= 8)
   int spl = 0;        // slots per lane V (WD_OPT_SLOTS_PER_LANE; 0 = from probe mode)
   int span = 0;       // windows per lane load S (WD_OPT_SPAN; 0 = auto)
+  int slices = 0;     // table slices of a grouped bulk insert (WD_OPT_SLICES; 0 = auto)
   // wd::kF_* kernel variants (WD_OPT_KERNEL_FLAGS).  Default all three: atom.exch value
   // updates take hot (Zipf) keys from 0.5 to 6-8 G inserts/s (tools/flags_bench.py),
   // L1-allowed probe loads add ~15 % there; the scrambled query chunk order adds 22-40 % to
@@ -412,6 +420,9 @@ void shard_free(Shard& s) {
   if (s.s_d2h) cudaStreamSynchronize(s.s_d2h);
   free_exchange(s);
   free_staging(s);
+  if (s.sl_buf) cudaFree(s.sl_buf);
+  if (s.sl_meta) cudaFree(s.sl_meta);
+  if (s.sl_done) cudaEventDestroy(s.sl_done);
   if (s.slots) cudaFree(s.slots);
   if (s.counters) cudaFree(s.counters);
   for (int i = 0; i < kStage; ++i) {
@@ -678,12 +689,71 @@ wd_status_t probe_soa(wd_table* t, Shard& s, int op, const wd::InSoA& in, uint32
   return launch_probe<false>(t, s, in, wd::OutSoA{ov, of}, n, st);
 }
 
+// Table slices for a bulk insert of n device-resident pairs (WD_OPT_SLICES): 16 when the
+// table is HBM-sized (> 512 MB) and the call has >= 2^22 pairs, else 1 (plain launch).
+int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
+  if (op != OP_INSERT || t->serial || t->slices == 1) return 1;
+  if (t->slices > 1) return t->slices;
+  return (s.cap * sizeof(unsigned long long) > (512ull << 20) && n >= (1ull << 22)) ? 16 : 1;
+}
+
+// Slice-grouped bulk insert.  Each chunk of <= 2^26 pairs is grouped by the table slice of
+// its keys' first region (Line 5: h(k) is monotone in fmix32(k + seed), so slice j of nbk
+// holds the region starts [j nb / nbk, (j + 1) nb / nbk)): a histogram, a scan and the
+// multisplit kernel write the pairs slice by slice into a scratch buffer; then one probe
+// launch per slice inserts them.  Each launch works on 1/nbk of the table, which the L2
+// holds a good part of: dirty lines take several inserts before they are written back and
+// fewer window loads go to DRAM.  Measured on B200 (tools/slice_probe.py,
+// profiles/r01_slices.txt): 2^28 pairs, |g| = 16, alpha 0.95: 15.0 -> 20.9 G inserts/s
+// for the probe launches.  Results are those of one launch: the probing of every key is
+// Fig. 3's; only the order in which the keys of one call are inserted changes (C20: any of
+// a call's duplicate values may win).
+wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStream_t st) {
+  constexpr uint64_t kChunkPairs = 1ull << 26;
+  const uint64_t cap = std::min<uint64_t>(io.n, kChunkPairs);
+  if (!s.sl_done) CK(cudaEventCreateWithFlags(&s.sl_done, cudaEventDisableTiming));
+  if (s.sl_used) CK(cudaStreamWaitEvent(st, s.sl_done, 0));   // scratch of an earlier call
+  if (s.sl_cap < cap) {
+    CK(cudaDeviceSynchronize());
+    if (s.sl_buf) cudaFree(s.sl_buf);
+    s.sl_buf = nullptr;
+    s.sl_cap = 0;
+    CK(cudaMalloc(&s.sl_buf, cap * sizeof(unsigned long long)));
+    s.sl_cap = cap;
+  }
+  if (!s.sl_meta) CK(cudaMalloc(&s.sl_meta, 97 * sizeof(unsigned long long)));
+  unsigned long long* counts = s.sl_meta;
+  unsigned long long* bounds = s.sl_meta + 32;
+  unsigned long long* cursor = s.sl_meta + 65;
+  wd::DstPtrs dst{};
+  for (int d = 0; d < nbk; ++d) dst.p[d] = s.sl_buf;
+  const int ms_grid_cap = t->sm_count * blocks_per_sm(wd::multisplit_kernel<true>);
+  for (uint64_t off = 0; off < io.n; off += kChunkPairs) {
+    const uint64_t cnt = std::min(kChunkPairs, io.n - off);
+    CK(cudaMemsetAsync(counts, 0, nbk * sizeof(unsigned long long), st));
+    wd::slice_hist_kernel<<<t->sm_count * 4, wd::kBlock, 0, st>>>(io.keys + off, cnt, nbk, s.hseed, counts);
+    wd::slice_scan_kernel<<<1, 32, 0, st>>>(counts, nbk, bounds, cursor);
+    const uint64_t tiles = (cnt + wd::kMsTile - 1) / wd::kMsTile;
+    wd::multisplit_kernel<true><<<int(std::min<uint64_t>(tiles, uint64_t(ms_grid_cap))), wd::kBlock, 0, st>>>(
+        io.keys + off, io.vals + off, cnt, dst, cursor, nullptr, nbk, s.hseed, 0, cnt, s.counters);
+    CK(cudaGetLastError());
+    t->launches += 3;
+    for (int j = 0; j < nbk; ++j)
+      TRY(launch_probe<true>(t, s, wd::InBucket{s.sl_buf, bounds, j}, wd::OutNone{}, cnt, st));
+  }
+  CK(cudaEventRecord(s.sl_done, st));
+  s.sl_used = true;
+  return WD_OK;
+}
+
 wd_status_t single_op(wd_table* t, int op, const IO& io, cudaStream_t stream) {
   const bool insert = op == OP_INSERT;
   Shard& s = t->local[0];
   DeviceGuard g(s.device);
   if (!needs_staging(io)) {  // device-resident: one kernel on the caller's stream
     if (io.n == 0) return WD_OK;
+    const int nbk = choose_slices(t, s, op, io.n);
+    if (nbk > 1) return slice_insert(t, s, io, nbk, stream);
     const wd::InSoA in{io.keys, io.vals, io.n};
     return probe_soa(t, s, op, in, io.vout, io.fout, io.n, stream);
   }
@@ -1325,6 +1395,10 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       if (v < 0 || v > 2) return fail(WD_ERR_INVALID_ARG, "span %lld", (long long)v);
       t->span = int(v);
       return WD_OK;
+    case WD_OPT_SLICES:
+      if (v < 0 || v > wd::kMaxShards) return fail(WD_ERR_INVALID_ARG, "slices %lld", (long long)v);
+      t->slices = int(v);
+      return WD_OK;
     default: return fail(WD_ERR_INVALID_ARG, "option %d is read-only or unknown", int(opt));
   }
 }
@@ -1345,6 +1419,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_SLOTS_PER_LANE: return t->spl;
     case WD_OPT_PART_MODE: return t->pmode;
     case WD_OPT_SPAN: return t->span;
+    case WD_OPT_SLICES: return t->slices;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;
     case WD_OPT_LOCAL_SHARDS: return int64_t(t->local.size());

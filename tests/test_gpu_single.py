@@ -442,3 +442,71 @@ def test_span_read_ahead(wd, G, span):
     cv, cf = oracle.expected_unique(q, n, 53, 54)
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
     assert np.array_equal(df.cpu().numpy().astype(bool), cf[: n // 2].astype(bool))
+
+
+@pytest.mark.parametrize("G", [4, 16])
+@pytest.mark.parametrize("slices", [1, 2, 16, 32])
+def test_slice_grouped_insert(wd, G, slices):
+    # WD_OPT_SLICES: a bulk insert grouped by table slice of the first region and inserted
+    # with one launch per slice.  Unique keys: exact map; duplicates with a reserved key:
+    # v in V(k), size = #distinct, the reserved key counted and never stored; a later
+    # stream-ordered call still wins.  (Grouping changes the order in which one call's keys
+    # are inserted, so only the map is compared, as for any concurrent call.)
+    n = 300_007
+    keys, vals = wdgen.unique_keys(n, 61), wdgen.values(n, 62)
+    q = wdgen.interleaved_queries(n, 61)
+    with wd.Table(capacity_for(n, 0.95), 1, G) as t:
+        t.set_option(wd.WD_OPT_SLICES, slices)
+        assert t.get_option(wd.WD_OPT_SLICES) == slices
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0 and t.size() == n
+    cv, cf = oracle.expected_unique(q, n, 61, 62)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+    nd = 400_000
+    dk = wdgen.uniform_keys(nd, 63) % np.uint32(150_000)
+    dk[::1000] = 0xFFFFFFFF                                  # reserved key (C8)
+    dv = wdgen.values(nd, 64)
+    with wd.Table(capacity_for(150_000, 0.9), 1, G) as t:
+        t.set_option(wd.WD_OPT_SLICES, slices)
+        t.insert(to_dev(dk), to_dev(dv))
+        assert t.sync() == wd.WD_ERR_RESERVED_KEY
+        assert t.counters()["reserved"] == 400
+        qq = np.arange(160_000, dtype=np.uint32)
+        ov, of = t.retrieve(to_dev(qq))
+        gv, gf = from_dev(ov), of.cpu().numpy()
+        m = oracle.Map(nd, dup_mode=True)
+        m.insert(dk, dv)
+        assert t.size() == m.size()
+        ev, ef = m.retrieve(qq)
+        assert np.array_equal(gf, ef)
+        assert np.all(m.pair_status(qq[gf == 1], gv[gf == 1]) >= 1)
+        k2 = np.unique(dk[dk != 0xFFFFFFFF])[:1000]
+        v2 = wdgen.values(k2.size, 65)
+        t.insert(to_dev(k2), to_dev(v2))
+        ov, of = t.retrieve(to_dev(k2))
+        assert np.array_equal(from_dev(ov), v2)
+
+
+def test_slice_grouped_insert_chunks(wd):
+    # more than one 2^26-pair chunk (auto slices on an HBM-sized table), ragged tail;
+    # every query checked against the closed form on a sample
+    import torch
+    import wdgen.gpu as gg
+    n, ks, vs = (1 << 26) * 2 + 12_345, 71, 72
+    keys, vals = gg.unique_keys(n, ks), gg.values(n, vs)
+    with wd.Table(capacity_for(n, 0.95), 1, 16) as t:
+        assert t.get_option(wd.WD_OPT_SLICES) == 0                 # auto -> 16 here
+        t.insert(keys, vals)
+        del vals
+        q = gg.interleaved_queries(n, ks, start=n - (1 << 24), count=1 << 25)
+        ov, of = t.retrieve(q)
+        assert t.sync() == 0 and t.size() == n
+        torch.cuda.synchronize()
+        rng = np.random.default_rng(1)
+        ii = torch.from_numpy(np.sort(rng.choice(q.numel(), 1 << 21, replace=False))).cuda()
+        qs = q[ii].cpu().numpy().view(np.uint32)
+        gv = ov[ii].cpu().numpy().view(np.uint32)
+        gf = of[ii].cpu().numpy()
+        assert t.launches >= 2 * (3 + 16)                             # two sliced chunks
+    cv, cf = oracle.expected_unique(qs, n, ks, vs)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
