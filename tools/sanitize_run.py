@@ -15,6 +15,9 @@ for G, V in [(4, 1), (8, 4), (4, 4), (1, 1), (2, 2), (16, 8), (32, 8)]:  # (1,1)
     with wd.Table(capacity_for(n, 0.9), 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
         check(*gpu_roundtrip(t, keys, vals, q))
+with wd.Table(capacity_for(n, 0.9), 1, 16) as t:   # slice-grouped bulk insert (forced)
+    t.set_option(wd.WD_OPT_SLICES, 16)
+    check(*gpu_roundtrip(t, keys, vals, q))
 with wd.Table(capacity_for(n, 0.9), 1, 4) as t:
     t.set_option(wd.WD_OPT_SERIAL, 1)
     check(*gpu_roundtrip(t, keys, vals, q))
