@@ -14,11 +14,15 @@ value      = (inserts + queries of all ranks) / max-over-ranks step time, device
              inputs, CUDA events on the launching stream.
 e2e        = the same step through the C-ABI with PINNED HOST buffers: H2D of keys/values/
              queries and D2H of values/found inside the timed region (out-of-core path a11).
-roofline   = the dominant kernel (per-launch CUDA-event time inside the timed region)
-             against the measured HBM copy bandwidth (MEASURED_PEAKS.json), with the
-             ALGORITHMIC bytes of SURVEY §8(d): insert 8 + 32 S_ins + 32 B, hit query
-             9 + 32 S_hit B, S from the oracle's sequential Fig. 3 replay
-             (tests/golden/probe_cost.json, written by tools/probe_cost.py).
+roofline   = the dominant call (CUDA-event time inside the timed region; the retrieve is
+             one probe launch, the bulk insert one launch per table slice plus the slice
+             grouping, WD_OPT_SLICES) against the measured HBM copy bandwidth
+             (MEASURED_PEAKS.json), with the ALGORITHMIC bytes of SURVEY §8(d): insert
+             8 + 32 S_ins + 32 B, hit query 9 + 32 S_hit B, S from the oracle's sequential
+             Fig. 3 replay (tests/golden/probe_cost.json, written by tools/probe_cost.py);
+             `traffic` = measured DRAM bytes per call (profiles/traffic.json, ncu), and
+             `pattern_ceiling` = the same call against this B200's measured random-access
+             rate for the probe's access pattern (profiles/ceilings.json).
 cpu_baseline = the oracle (single-threaded C dictionary) on a bounded sample.
 """
 from __future__ import annotations
