@@ -1,0 +1,8 @@
+// probe_g1.cu — the probe-kernel dispatch for |g| = 1 (see wd_host.cuh): one
+// translation unit per group size so the build compiles them in parallel.
+#define WD_PROBE_TU 1
+#include "wd_host.cuh"
+
+namespace wdi {
+WD_PROBE_COMBOS(WD_PROBE_INST, 1)
+}  // namespace wdi

@@ -1,0 +1,8 @@
+// probe_g4.cu — the probe-kernel dispatch for |g| = 4 (see wd_host.cuh): one
+// translation unit per group size so the build compiles them in parallel.
+#define WD_PROBE_TU 4
+#include "wd_host.cuh"
+
+namespace wdi {
+WD_PROBE_COMBOS(WD_PROBE_INST, 4)
+}  // namespace wdi
