@@ -67,6 +67,10 @@ typedef enum {
 /* ------------------------------------------------------------------ creation ------- */
 
 /* Single process.  n_gpus == 1: one table on the current CUDA device.
+ * Side effect: while any table lives on a device, that device's L2 fetch granularity
+ * (cudaLimitMaxL2FetchGranularity, device-wide) is 32 B so random 32-B windows do not pull
+ * whole lines; the caller's value is restored when the last table on the device is
+ * destroyed (environment WD_L2_FETCH_BYTES=<bytes> overrides, 0 = leave it alone).
  * n_gpus > 1: one shard per device 0..n_gpus-1, keys owned by shard p(k),
  * peer access over NVLink; host input is split into n_gpus contiguous chunks.
  * capacity: total slots c (alpha = n / c).  Each shard gets ceil(c / m) slots,
@@ -102,7 +106,10 @@ wd_status_t wd_rank_handle(wd_table_t* t, uint8_t out[WD_RANK_HANDLE_BYTES]);
 wd_status_t wd_rank_connect(wd_table_t* t, const uint8_t* handles, wd_allreduce_fn allreduce,
                             void* ctx);
 
-/* NULL-safe.  Synchronizes, then frees table, buffers, peer mappings and communicators. */
+/* Resource release (no passage of the paper: its table lives for the whole run).
+ * NULL-safe.  Synchronizes the table's devices, then frees the table, staging and scratch
+ * buffers, peer mappings and communicators; in rank mode it is collective (a barrier
+ * before unmapping).  Errors are ignored. */
 void wd_destroy(wd_table_t* t);
 
 /* ------------------------------------------------------------------ the hot path --- */
@@ -117,10 +124,14 @@ wd_status_t wd_clear(wd_table_t* t, wd_stream_t stream);
 wd_status_t wd_insert(wd_table_t* t, const uint32_t* keys, const uint32_t* vals, uint64_t n,
                       wd_stream_t stream);
 
-/* a4 (and a6-a10 when m > 1, a11 for host pointers): for each i, found_out[i] = 1 and
- * vals_out[i] = the stored value if keys[i] is present, else found_out[i] = 0 and
- * vals_out[i] = WD_NOT_FOUND.  Results in input order.  vals_out may be NULL (presence
- * only); found_out may be NULL. */
+/* a4 — retrieval "in a similar way" to the insertion: the same windows of the same
+ * region sequence; a query stops at the first window holding its key (found) or an empty
+ * slot (absent, reading C10).  With m > 1 also a6-a10: multisplit -> transposition ->
+ * local query -> reverse transposition; with host pointers a11.
+ * For each i: found_out[i] = 1 and vals_out[i] = the stored value if keys[i] is present,
+ * else found_out[i] = 0 and vals_out[i] = WD_NOT_FOUND (C11).  keys: uint32[n];
+ * vals_out: uint32[n] or NULL (presence only); found_out: uint8[n] or NULL.  Results in
+ * input order.  The reserved key reports not-found (sticky WD_ERR_RESERVED_KEY). */
 wd_status_t wd_retrieve(wd_table_t* t, const uint32_t* keys, uint32_t* vals_out,
                         uint8_t* found_out, uint64_t n, wd_stream_t stream);
 
@@ -134,11 +145,14 @@ wd_status_t wd_erase(wd_table_t* t, const uint32_t* keys, uint8_t* found_out, ui
 
 /* P:63 reconstruction: re-insert every live entry into a fresh table of the same capacity
  * with the hash seed `seed` (translated variants h(k + seed)); tombstones are dropped.
- * Synchronizes; needs a second table's worth of device memory transiently. */
+ * Synchronizes.  Needs, transiently, a second table's worth of device memory plus 8 B per
+ * live entry; on any failure the old table is kept and nothing leaks.  Sticky error
+ * counters (TABLE_FULL / RESERVED_KEY / EXCHANGE) survive the rebuild. */
 wd_status_t wd_rebuild(wd_table_t* t, uint32_t seed, wd_stream_t stream);
 
-/* a5: number of distinct keys stored (summed over shards and ranks).  Synchronizes.
- * UINT64_MAX on error. */
+/* a5: number of distinct keys stored (summed over shards and ranks) — the n of the load
+ * factor alpha = n / c.  Synchronizes (collective in rank mode).  UINT64_MAX on
+ * error (wd_last_error). */
 uint64_t wd_size(wd_table_t* t);
 
 /* physical slots summed over all shards (load = wd_size / wd_capacity). */
@@ -188,9 +202,12 @@ typedef enum {
                                 is grouped by table slice of the keys' first region (Line 5) and
                                 inserted with one probe launch per slice (better L2 reuse); the
                                 probing of each key is unchanged.  0 (default): 16 slices for
-                                tables > 512 MB and calls of >= 2^22 pairs, else 1 (off);
+                                tables > 512 MB and calls of >= 2^26 pairs (unless the span
+                                read-ahead applies), else 1 (off);
                                 1: off; 2..32: that many slices.  Uses 8 B of scratch per pair,
-                                at most 2^26 pairs at a time. */
+                                at most 2^26 pairs at a time, kept for the table's lifetime
+                                (stream-ordered allocation); in auto mode a failed scratch
+                                allocation falls back to the plain launch. */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -108,18 +108,32 @@ def _check(status: int):
         raise WarpDriveError(status, _lib.wd_last_error_message().decode())
 
 
-def _addr(x):
-    """(pointer, nelem, is_cuda) of a torch tensor / numpy array / None."""
+def _addr(x, itemsize: int | None = None, what: str = "buffer", min_len: int | None = None):
+    """(pointer, nelem, is_cuda) of a torch tensor / numpy array / None.  The C-ABI takes
+    uint32 keys / values and uint8 found flags: `itemsize` is checked (any 4-byte integer
+    dtype is reinterpreted bit for bit; int64 or 1-2-byte keys would be misread), and an
+    output must hold at least `min_len` elements."""
     if x is None:
         return None, 0, False
     if isinstance(x, np.ndarray):
-        assert x.flags.c_contiguous
-        return x.ctypes.data, x.size, False
-    import torch
-    if isinstance(x, torch.Tensor):
-        assert x.is_contiguous()
-        return x.data_ptr(), x.numel(), x.is_cuda
-    raise TypeError(f"unsupported buffer type {type(x)}")
+        if not x.flags.c_contiguous:
+            raise ValueError(f"{what}: must be C-contiguous")
+        if itemsize is not None and (x.dtype.itemsize != itemsize or x.dtype.kind not in "iu"):
+            raise TypeError(f"{what}: need a {itemsize}-byte integer dtype, got {x.dtype}")
+        p, n, cuda = x.ctypes.data, x.size, False
+    else:
+        import torch
+        if not isinstance(x, torch.Tensor):
+            raise TypeError(f"unsupported buffer type {type(x)}")
+        if not x.is_contiguous():
+            raise ValueError(f"{what}: must be contiguous")
+        if itemsize is not None and (x.element_size() != itemsize or x.dtype.is_floating_point
+                                     or x.dtype.is_complex or x.dtype == torch.bool):
+            raise TypeError(f"{what}: need a {itemsize}-byte integer dtype, got {x.dtype}")
+        p, n, cuda = x.data_ptr(), x.numel(), x.is_cuda
+    if min_len is not None and n < min_len:
+        raise ValueError(f"{what}: {n} elements, need at least {min_len}")
+    return p, n, cuda
 
 
 def _stream(stream, dev_hint=None):
@@ -199,14 +213,14 @@ class Table:
         _check(_lib.wd_clear(self._h, _stream(stream)))
 
     def insert(self, keys, vals, stream=None):
-        kp, n, kc = _addr(keys)
-        vp, nv, vc = _addr(vals)
+        kp, n, kc = _addr(keys, 4, "keys")
+        vp, nv, vc = _addr(vals, 4, "vals")
         if n != nv:
             raise ValueError("keys and vals differ in length")
         _check(_lib.wd_insert(self._h, kp, vp, n, _stream(stream)))
 
     def retrieve(self, keys, vals_out=None, found_out=None, stream=None):
-        kp, n, kc = _addr(keys)
+        kp, n, kc = _addr(keys, 4, "keys")
         if vals_out is None and found_out is None:
             import torch
             dev = keys.device if isinstance(keys, torch.Tensor) else None
@@ -217,14 +231,14 @@ class Table:
             else:
                 vals_out = np.empty(n, np.uint32)
                 found_out = np.empty(n, np.uint8)
-        vp, _, _ = _addr(vals_out)
-        fp, _, _ = _addr(found_out)
+        vp, _, _ = _addr(vals_out, 4, "vals_out", n)
+        fp, _, _ = _addr(found_out, 1, "found_out", n)
         _check(_lib.wd_retrieve(self._h, kp, vp, fp, n, _stream(stream)))
         return vals_out, found_out
 
     def erase(self, keys, found_out=None, stream=None):
         """P:91 deletion; found_out[i] = 1 for the occurrence that removed keys[i]."""
-        kp, n, kc = _addr(keys)
+        kp, n, kc = _addr(keys, 4, "keys")
         if found_out is None:
             import torch
             if isinstance(keys, torch.Tensor):
@@ -232,7 +246,7 @@ class Table:
                 found_out = torch.empty(n, dtype=torch.uint8, device=keys.device, pin_memory=pin)
             else:
                 found_out = np.empty(n, np.uint8)
-        fp, _, _ = _addr(found_out)
+        fp, _, _ = _addr(found_out, 1, "found_out", n)
         _check(_lib.wd_erase(self._h, kp, fp, n, _stream(stream)))
         return found_out
 

@@ -17,6 +17,8 @@
 // =====================================================================================
 #include "wd_host.cuh"
 
+#include <mutex>
+
 namespace wdi {
 
 thread_local wd_status_t g_last = WD_OK;
@@ -31,17 +33,46 @@ wd_status_t fail(wd_status_t s, const char* fmt, ...) {
   return s;
 }
 
+// ------------------------------------------------------------------ L2 fetch granularity
+// Random 32-byte windows: do not let L2 promote a sector miss to a 64/128-byte DRAM fetch
+// (measured: 6.7 DRAM sectors per |g| = 4 insert with the default, 2.4 needed).  The limit
+// is device-wide, so it is scoped to the tables' lifetime: the first live shard on a device
+// records the caller's value and sets 32 B; the last one destroyed restores it
+// (include/warpdrive.h, wd_create).  WD_L2_FETCH_BYTES=<bytes> overrides, 0 leaves it alone.
+struct L2Hold { int users = 0; size_t saved = 0; bool set = false; };
+L2Hold g_l2[64];
+std::mutex g_l2_mu;
+
+wd_status_t l2_fetch_acquire(int device) {
+  std::lock_guard<std::mutex> lk(g_l2_mu);
+  if (device < 0 || device >= 64) return WD_OK;
+  L2Hold& h = g_l2[device];
+  if (h.users++ > 0) return WD_OK;
+  size_t want = 32;
+  if (const char* e = getenv("WD_L2_FETCH_BYTES")) want = size_t(atoi(e));
+  h.set = false;
+  if (want == 0) return WD_OK;
+  CK(cudaDeviceGetLimit(&h.saved, cudaLimitMaxL2FetchGranularity));
+  CK(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, want));
+  h.set = true;
+  return WD_OK;
+}
+void l2_fetch_release(int device) {
+  std::lock_guard<std::mutex> lk(g_l2_mu);
+  if (device < 0 || device >= 64) return;
+  L2Hold& h = g_l2[device];
+  if (h.users <= 0 || --h.users > 0) return;
+  if (h.set && cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, h.saved) != cudaSuccess)
+    cudaGetLastError();
+  h.set = false;
+}
+
 // ------------------------------------------------------------------ shard lifetime
 wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
                        cudaStream_t shared_main) {
   DeviceGuard g(device);
-  // Random 32-byte windows: do not let L2 promote a sector miss to a 64/128-byte DRAM
-  // fetch (measured: 6.7 DRAM sectors per insert with the default, 2.4 needed).
-  if (const char* e = getenv("WD_L2_FETCH_BYTES")) {
-    if (atoi(e) > 0) CK(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, size_t(atoi(e))));
-  } else {
-    CK(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, 32));
-  }
+  TRY(l2_fetch_acquire(device));
+  s.l2_held = true;
   s.id = id;
   s.device = device;
   if (cap == 0) return fail(WD_ERR_INVALID_ARG, "capacity per shard exceeds 4 * 2^32 slots");
@@ -132,6 +163,7 @@ void shard_free(Shard& s) {
   if (s.ev_join_h2d) cudaEventDestroy(s.ev_join_h2d);
   if (s.ev_join_d2h) cudaEventDestroy(s.ev_join_d2h);
   if (s.ev_join_probe) cudaEventDestroy(s.ev_join_probe);
+  if (s.l2_held) l2_fetch_release(s.device);
   if (s.own_main && s.s_main) cudaStreamDestroy(s.s_main);
   if (s.own_main && s.s_probe) cudaStreamDestroy(s.s_probe);
   if (s.s_h2d) cudaStreamDestroy(s.s_h2d);
@@ -308,13 +340,20 @@ struct IO {
 // stage batch b's input of `io` into device memory; returns device pointers
 wd_status_t stage_in(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slot, bool with_vals,
                      const uint32_t** dk, const uint32_t** dv) {
+  DeviceGuard g(s.device);
+  // the slot's staging buffers (input and output) may still be used by an earlier batch —
+  // of this call or of an earlier call on any stream: both the copy-in and the kernel that
+  // writes the slot's outputs wait for its release
+  if (s.h2d_pending[slot]) {
+    CK(cudaStreamWaitEvent(s.s_h2d, s.ev_free[slot], 0));
+    CK(cudaStreamWaitEvent(s.s_main, s.ev_free[slot], 0));
+    s.h2d_pending[slot] = false;
+  }
   if (io.kin == PK_DEVICE) {
     *dk = io.keys + off;
     *dv = with_vals ? io.vals + off : nullptr;
     return WD_OK;
   }
-  DeviceGuard g(s.device);
-  if (s.h2d_pending[slot]) CK(cudaStreamWaitEvent(s.s_h2d, s.ev_free[slot], 0));
   const uint32_t* hk = io.keys + off;
   const uint32_t* hv = with_vals ? io.vals + off : nullptr;
   if (io.kin == PK_PAGEABLE && cnt) {
@@ -331,7 +370,6 @@ wd_status_t stage_in(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slo
   }
   CK(cudaEventRecord(s.ev_h2d[slot], s.s_h2d));
   CK(cudaStreamWaitEvent(s.s_main, s.ev_h2d[slot], 0));
-  s.h2d_pending[slot] = true;
   *dk = s.st_keys[slot];
   *dv = with_vals ? s.st_vals[slot] : nullptr;
   return WD_OK;
@@ -354,7 +392,10 @@ wd_status_t stage_out(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int sl
   DeviceGuard g(s.device);
   CK(cudaEventRecord(s.ev_kdone[slot], s.s_main));
   if (!query || io.kout == PK_DEVICE) {
-    if (io.kin != PK_DEVICE) CK(cudaEventRecord(s.ev_free[slot], s.s_main));
+    if (io.kin != PK_DEVICE) {
+      CK(cudaEventRecord(s.ev_free[slot], s.s_main));
+      s.h2d_pending[slot] = true;
+    }
     return WD_OK;
   }
   CK(cudaStreamWaitEvent(s.s_d2h, s.ev_kdone[slot], 0));
@@ -362,10 +403,12 @@ wd_status_t stage_out(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int sl
     if (io.vout && cnt) CK(cudaMemcpyAsync(io.vout + off, s.st_vout[slot], cnt * 4, cudaMemcpyDeviceToHost, s.s_d2h));
     if (io.fout && cnt) CK(cudaMemcpyAsync(io.fout + off, s.st_fout[slot], cnt, cudaMemcpyDeviceToHost, s.s_d2h));
     CK(cudaEventRecord(s.ev_free[slot], s.s_d2h));
+    s.h2d_pending[slot] = true;
   } else {
     if (io.vout && cnt) CK(cudaMemcpyAsync(s.pin_vout[slot], s.st_vout[slot], cnt * 4, cudaMemcpyDeviceToHost, s.s_d2h));
     if (io.fout && cnt) CK(cudaMemcpyAsync(s.pin_fout[slot], s.st_fout[slot], cnt, cudaMemcpyDeviceToHost, s.s_d2h));
     CK(cudaEventRecord(s.ev_free[slot], s.s_d2h));
+    s.h2d_pending[slot] = true;
     CK(cudaEventSynchronize(s.ev_free[slot]));
     if (io.vout) memcpy(io.vout + off, s.pin_vout[slot], cnt * 4);
     if (io.fout) memcpy(io.fout + off, s.pin_fout[slot], cnt);
@@ -388,10 +431,17 @@ wd_status_t probe_soa(wd_table* t, Shard& s, int op, const wd::InSoA& in, uint32
 
 // Table slices for a bulk insert of n device-resident pairs (WD_OPT_SLICES): 16 when the
 // table is HBM-sized (> 512 MB) and the call has >= 2^22 pairs, else 1 (plain launch).
+// Auto only where it was measured to pay (profiles/r01_slices.txt: 2^28 pairs into 2.3 GB;
+// 16 slices over 2^24-pair chunks were SLOWER than one launch): calls of >= 2^26 pairs, so
+// each slice launch gets >= 2^22 keys, and not where the plain launch uses the span
+// read-ahead (|g| = 1), whose gain the sliced launches (InBucket) do not have.
 int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
   if (op != OP_INSERT || t->serial || t->slices == 1) return 1;
   if (t->slices > 1) return t->slices;
-  return (s.cap * sizeof(unsigned long long) > (512ull << 20) && n >= (1ull << 22)) ? 16 : 1;
+  if (s.cap * sizeof(unsigned long long) <= (512ull << 20) || n < (1ull << 26)) return 1;
+  const int v = choose_v(t, s, t->G_used, true);
+  if (choose_span(t, s, t->G_used, v) == 2) return 1;
+  return 16;
 }
 
 // Slice-grouped bulk insert.  Each chunk of <= 2^26 pairs is grouped by the table slice of
@@ -411,11 +461,23 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
   if (!s.sl_done) CK(cudaEventCreateWithFlags(&s.sl_done, cudaEventDisableTiming));
   if (s.sl_used) CK(cudaStreamWaitEvent(st, s.sl_done, 0));   // scratch of an earlier call
   if (s.sl_cap < cap) {
-    CK(cudaDeviceSynchronize());
-    if (s.sl_buf) cudaFree(s.sl_buf);
+    // stream-ordered (no device synchronisation): the old scratch is released after its
+    // last use (st waits on sl_done above), the new one is allocated in st's order.  The
+    // scratch (8 B per pair, <= 512 MB) is kept for the table's lifetime.
+    if (s.sl_buf) CK(cudaFreeAsync(s.sl_buf, st));
     s.sl_buf = nullptr;
     s.sl_cap = 0;
-    CK(cudaMalloc(&s.sl_buf, cap * sizeof(unsigned long long)));
+    const cudaError_t e = cudaMallocAsync(&s.sl_buf, cap * sizeof(unsigned long long), st);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      s.sl_buf = nullptr;
+      if (t->slices == 0) {        // auto: the optimisation steps back, the call still runs
+        const wd::InSoA in{io.keys, io.vals, io.n};
+        return probe_soa(t, s, OP_INSERT, in, nullptr, nullptr, io.n, st);
+      }
+      return fail(e == cudaErrorMemoryAllocation ? WD_ERR_OUT_OF_MEMORY : WD_ERR_CUDA,
+                  "slice scratch of %llu pairs: %s", (unsigned long long)cap, cudaGetErrorString(e));
+    }
     s.sl_cap = cap;
   }
   if (!s.sl_meta) CK(cudaMalloc(&s.sl_meta, 97 * sizeof(unsigned long long)));
@@ -462,7 +524,6 @@ wd_status_t single_op(wd_table* t, int op, const IO& io, cudaStream_t stream) {
   TRY(ensure_staging(s, B, io.kin == PK_PAGEABLE || io.kout == PK_PAGEABLE));
   cudaEvent_t ev0;
   TRY(fork_from(t, stream, &ev0));
-  for (bool& p : s.h2d_pending) p = false;
   const uint64_t nbt = (io.n + B - 1) / B;
   for (uint64_t b = 0; b < nbt; ++b) {
     const int slot = int(b % kStage);
@@ -523,8 +584,6 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
   if (nbt == 0) return WD_OK;
   cudaEvent_t ev0;
   TRY(fork_from(t, stream, &ev0));
-  for (auto& s : t->local)
-    for (bool& p : s.h2d_pending) p = false;
 
   // Three phases per batch b (epoch e = epoch0 + 1 + b, exchange slot e % 2):
   //   A (s_main):  multisplit fused with the push into the owners' receive regions, then
@@ -989,30 +1048,61 @@ wd_status_t wd_rebuild(wd_table_t* t, uint32_t seed, wd_stream_t stream) {
   for (auto& s : t->local) {
     DeviceGuard g(s.device);
     CK(cudaStreamSynchronize(st));
-    CK(cudaDeviceSynchronize());
-    // 1. gather the live slots (the contents survive, tombstones do not)
+    CK(cudaStreamSynchronize(s.s_main));
+    CK(cudaStreamSynchronize(s.s_probe));
+    // live entries = new keys - erased keys (counters: the contents survive, the
+    // tombstones do not)
+    unsigned long long c[wd::CNT_N];
+    CK(cudaMemcpy(c, s.counters, sizeof c, cudaMemcpyDeviceToHost));
+    const uint64_t n_live = c[wd::CNT_NEW] - c[wd::CNT_ERASED];
     unsigned long long *live = nullptr, *cnt = nullptr, *fresh = nullptr;
-    CK(cudaMalloc(&live, s.cap * sizeof(unsigned long long)));
-    CK(cudaMalloc(&cnt, sizeof(unsigned long long)));
-    CK(cudaMalloc(&fresh, s.cap * sizeof(unsigned long long)));
-    CK(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long), s.s_main));
+    auto release = [&]() {
+      if (live) cudaFree(live);
+      if (cnt) cudaFree(cnt);
+      if (fresh) cudaFree(fresh);
+    };
+    cudaError_t e = cudaMalloc(&live, std::max<uint64_t>(n_live, 1) * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc(&cnt, sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMalloc(&fresh, s.cap * sizeof(unsigned long long));
+    if (e == cudaSuccess) e = cudaMemsetAsync(cnt, 0, sizeof(unsigned long long), s.s_main);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      release();
+      return fail(e == cudaErrorMemoryAllocation ? WD_ERR_OUT_OF_MEMORY : WD_ERR_CUDA,
+                  "wd_rebuild: %s", cudaGetErrorString(e));
+    }
+    // 1. gather the live slots; 2. a fresh table with the distinct hash (translated variant,
+    // P:161).  The sticky error counters are kept; only new / erased restart.
     const int cgrid = t->serial ? 1 : t->sm_count * 8;
-    wd::compact_kernel<<<cgrid, t->serial ? 32 : wd::kBlock, 0, s.s_main>>>(s.slots, s.cap, live, cnt);
-    CK(cudaGetLastError());
-    // 2. a fresh table with the distinct hash (translated variant)
-    wd::fill_kernel<<<t->sm_count * 4, wd::kBlock, 0, s.s_main>>>(fresh, s.cap, s.counters, wd::CNT_N);
-    CK(cudaGetLastError());
+    wd::compact_kernel<<<cgrid, t->serial ? 32 : wd::kBlock, 0, s.s_main>>>(s.slots, s.cap, live, n_live, cnt);
+    wd::fill_kernel<<<t->sm_count * 4, wd::kBlock, 0, s.s_main>>>(fresh, s.cap, s.counters, 0);
+    e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaMemsetAsync(s.counters + wd::CNT_NEW, 0, sizeof(unsigned long long), s.s_main);
+    if (e == cudaSuccess) e = cudaMemsetAsync(s.counters + wd::CNT_ERASED, 0, sizeof(unsigned long long), s.s_main);
+    if (e != cudaSuccess) {
+      cudaStreamSynchronize(s.s_main);
+      release();
+      return fail(WD_ERR_CUDA, "wd_rebuild: %s", cudaGetErrorString(e));
+    }
     t->launches += 2;
+    // 3. re-insert (Fig. 3) from the gathered pairs into the fresh slots
     unsigned long long* old = s.slots;
+    const uint32_t old_seed = s.hseed;
     s.slots = fresh;
     s.hseed = seed;
-    // 3. re-insert (Fig. 3) from the gathered pairs
-    const wd::InSeg<true> in{live, cnt, s.cap, 1};
-    TRY(launch_probe<true>(t, s, in, wd::OutNone{}, s.cap, s.s_main));
-    CK(cudaStreamSynchronize(s.s_main));
+    const wd::InSeg<true> in{live, cnt, std::max<uint64_t>(n_live, 1), 1};
+    wd_status_t r = launch_probe<true>(t, s, in, wd::OutNone{}, n_live, s.s_main);
+    e = cudaStreamSynchronize(s.s_main);
+    if (r != WD_OK || e != cudaSuccess) {   // keep the old table
+      s.slots = old;
+      s.hseed = old_seed;
+      release();
+      if (r == WD_OK) r = fail(WD_ERR_CUDA, "wd_rebuild: %s", cudaGetErrorString(e));
+      return r;
+    }
+    fresh = nullptr;                         // now the table
     cudaFree(old);
-    cudaFree(live);
-    cudaFree(cnt);
+    release();
   }
   return WD_OK;
 }

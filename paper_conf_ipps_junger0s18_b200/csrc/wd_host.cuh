@@ -106,7 +106,8 @@ struct Shard {
   cudaEvent_t ev_h2d[kStage] = {}, ev_free[kStage] = {}, ev_kdone[kStage] = {}, ev_d2h[kStage] = {};
   cudaEvent_t ev_join_main = nullptr, ev_join_h2d = nullptr, ev_join_d2h = nullptr;
   cudaEvent_t ev_join_probe = nullptr;
-  bool h2d_pending[kStage] = {}, d2h_pending[kStage] = {};
+  bool h2d_pending[kStage] = {};   // the slot's staging buffers have a pending release (ev_free)
+  bool l2_held = false;            // holds the device's L2 fetch-granularity setting
 };
 
 }  // namespace wdi

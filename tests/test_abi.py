@@ -75,3 +75,25 @@ def test_oracle_and_generator_libraries_load():
     build.build()
     g = ctypes.CDLL(build.GENLIB)
     assert hasattr(g, "wdgen_unique_keys")
+
+
+def test_binding_checks_dtypes_and_lengths(lib):
+    # the binding must refuse buffers the C-ABI would misread (int64 / 1-2-byte
+    # keys, float values, short outputs) instead of passing their bytes through
+    import numpy as np
+    import torch
+    import paper_conf_ipps_junger0s18_b200 as wd
+    a = wd._addr
+    assert a(np.zeros(8, np.uint32), 4, "keys")[1] == 8
+    assert a(torch.zeros(8, dtype=torch.int32), 4, "keys")[1] == 8
+    assert a(torch.zeros(8, dtype=torch.uint8), 1, "found_out", 8)[1] == 8
+    for bad in (np.zeros(8, np.int64), np.zeros(8, np.uint16), np.zeros(8, np.float32),
+                torch.arange(8), torch.zeros(8, dtype=torch.float32)):
+        with pytest.raises(TypeError):
+            a(bad, 4, "keys")
+    with pytest.raises(TypeError):
+        a(torch.zeros(8, dtype=torch.bool), 1, "found_out")
+    with pytest.raises(ValueError):
+        a(np.zeros(7, np.uint32), 4, "vals_out", 8)
+    with pytest.raises(ValueError):
+        a(np.zeros((4, 4), np.uint32)[:, 0], 4, "keys")

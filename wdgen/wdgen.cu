@@ -128,6 +128,9 @@ int grid_for(uint64_t n) {
 
 extern "C" {
 int wdgen_unique_keys(uint32_t* out, uint64_t start, uint64_t n, uint64_t seed, cudaStream_t st) {
+  // pi_s is a bijection on [0, 2^32 - 1) only (the sentinel is cycle-walked out, C14):
+  // index 2^32 - 1 would alias another key
+  if (start > uint64_t(kEmpty) || n > uint64_t(kEmpty) - start) return int(cudaErrorInvalidValue);
   if (n) k_unique<<<grid_for(n), 256, 0, st>>>(out, start, n, round_keys(seed));
   return int(cudaGetLastError());
 }
@@ -141,6 +144,9 @@ int wdgen_uniform_keys(uint32_t* out, uint64_t start, uint64_t n, uint64_t seed,
 }
 int wdgen_interleaved_queries(uint32_t* out, uint64_t n_present, uint64_t start, uint64_t count,
                               uint64_t seed, cudaStream_t st) {
+  const uint64_t jmax = start + count;   // largest index used: (jmax - 1) / 2 + n_present
+  if (count && (count > (1ull << 33) || (jmax - 1) / 2 + n_present >= uint64_t(kEmpty)))
+    return int(cudaErrorInvalidValue);
   if (count) k_interleaved<<<grid_for(count), 256, 0, st>>>(out, n_present, start, count, round_keys(seed));
   return int(cudaGetLastError());
 }
