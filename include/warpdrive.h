@@ -135,6 +135,22 @@ wd_status_t wd_insert(wd_table_t* t, const uint32_t* keys, const uint32_t* vals,
 wd_status_t wd_retrieve(wd_table_t* t, const uint32_t* keys, uint32_t* vals_out,
                         uint8_t* found_out, uint64_t n, wd_stream_t stream);
 
+/* The paper's device-sided cascades: the call's pairs are
+ * already split into per-GPU portions in device memory.  Arrays have one entry per
+ * LOCAL shard (wd_get_option(WD_OPT_LOCAL_SHARDS): n_gpus for wd_create / loopback tables,
+ * 1 in rank mode); keys[r] / vals[r] (uint32[n[r]]) live on shard r's device (host memory is
+ * also accepted and streamed, a11); streams[r] is a stream of that device (NULL array: the
+ * legacy stream everywhere).  Each portion is multisplit and sent to its owners exactly like
+ * the whole-table calls; completion of shard r's part (its table's inserts, or the results of
+ * its portion's queries) is ordered on streams[r].  Same semantics and errors as
+ * wd_insert / wd_retrieve. */
+wd_status_t wd_insert_sharded(wd_table_t* t, const uint32_t* const keys[],
+                              const uint32_t* const vals[], const uint64_t n[],
+                              const wd_stream_t streams[]);
+wd_status_t wd_retrieve_sharded(wd_table_t* t, const uint32_t* const keys[],
+                                uint32_t* const vals_out[], uint8_t* const found_out[],
+                                const uint64_t n[], const wd_stream_t streams[]);
+
 /* P:91 deletion (NEXT #3; barrier-separated from inserts, i.e. not concurrent with a
  * wd_insert on the same table): every present key in keys[0..n) is removed — its slot
  * becomes a tombstone (reading C9': probed past by queries, not reused by inserts until

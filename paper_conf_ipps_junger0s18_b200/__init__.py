@@ -43,7 +43,7 @@ EXPORTS = ["wd_create", "wd_create_loopback", "wd_create_rank", "wd_rank_handle"
            "wd_destroy", "wd_clear", "wd_insert", "wd_retrieve", "wd_size", "wd_capacity",
            "wd_sync", "wd_set_option", "wd_get_option", "wd_last_error", "wd_error_string",
            "wd_last_error_message", "wd_shard_capacity", "wd_dump", "wd_counters", "wd_erase",
-           "wd_rebuild"]
+           "wd_rebuild", "wd_insert_sharded", "wd_retrieve_sharded"]
 
 
 class WarpDriveError(RuntimeError):
@@ -88,6 +88,8 @@ def _load():
         "wd_counters": ([p, i32, p], i32),
         "wd_erase": ([p, p, p, u64, p], i32),
         "wd_rebuild": ([p, C.c_uint32, p], i32),
+        "wd_insert_sharded": ([p, p, p, p, p], i32),
+        "wd_retrieve_sharded": ([p, p, p, p, p, p], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -234,6 +236,36 @@ class Table:
         vp, _, _ = _addr(vals_out, 4, "vals_out", n)
         fp, _, _ = _addr(found_out, 1, "found_out", n)
         _check(_lib.wd_retrieve(self._h, kp, vp, fp, n, _stream(stream)))
+        return vals_out, found_out
+
+    def _local(self):
+        return self.get_option(WD_OPT_LOCAL_SHARDS)
+
+    def insert_sharded(self, keys, vals, streams=None):
+        """Device-sided cascade: keys[r] / vals[r] are local shard r's
+        portion, on its device; streams[r] (optional) is a stream of that device."""
+        L = self._local()
+        if len(keys) != L or len(vals) != L:
+            raise ValueError(f"need {L} portions (one per local shard)")
+        kp = (C.c_void_p * L)(*[_addr(k, 4, "keys")[0] for k in keys])
+        vp = (C.c_void_p * L)(*[_addr(v, 4, "vals")[0] for v in vals])
+        ns = [_addr(k, 4)[1] for k in keys]
+        if ns != [_addr(v, 4)[1] for v in vals]:
+            raise ValueError("keys and vals differ in length")
+        n = (C.c_uint64 * L)(*ns)
+        sp = (C.c_void_p * L)(*[_stream(x) for x in streams]) if streams is not None else None
+        _check(_lib.wd_insert_sharded(self._h, kp, vp, n, sp))
+
+    def retrieve_sharded(self, keys, vals_out, found_out, streams=None):
+        L = self._local()
+        if not (len(keys) == len(vals_out) == len(found_out) == L):
+            raise ValueError(f"need {L} portions (one per local shard)")
+        ns = [_addr(k, 4)[1] for k in keys]
+        kp = (C.c_void_p * L)(*[_addr(k, 4, "keys")[0] for k in keys])
+        vp = (C.c_void_p * L)(*[_addr(v, 4, "vals_out", n)[0] for v, n in zip(vals_out, ns)])
+        fp = (C.c_void_p * L)(*[_addr(f, 1, "found_out", n)[0] for f, n in zip(found_out, ns)])
+        sp = (C.c_void_p * L)(*[_stream(x) for x in streams]) if streams is not None else None
+        _check(_lib.wd_retrieve_sharded(self._h, kp, vp, fp, (C.c_uint64 * L)(*ns), sp))
         return vals_out, found_out
 
     def erase(self, keys, found_out=None, stream=None):

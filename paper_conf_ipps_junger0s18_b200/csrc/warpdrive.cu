@@ -99,6 +99,7 @@ wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
   CK(cudaEventCreateWithFlags(&s.ev_join_h2d, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&s.ev_join_d2h, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&s.ev_join_probe, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&s.ev_fork, cudaEventDisableTiming));
   // a1: fresh table
   const int grid = t->sm_count * 4;
   wd::fill_kernel<<<grid, wd::kBlock, 0, s.s_main>>>(s.slots, s.cap, s.counters, wd::CNT_N);
@@ -163,6 +164,7 @@ void shard_free(Shard& s) {
   if (s.ev_join_h2d) cudaEventDestroy(s.ev_join_h2d);
   if (s.ev_join_d2h) cudaEventDestroy(s.ev_join_d2h);
   if (s.ev_join_probe) cudaEventDestroy(s.ev_join_probe);
+  if (s.ev_fork) cudaEventDestroy(s.ev_fork);
   if (s.l2_held) l2_fetch_release(s.device);
   if (s.own_main && s.s_main) cudaStreamDestroy(s.s_main);
   if (s.own_main && s.s_probe) cudaStreamDestroy(s.s_probe);
@@ -295,33 +297,47 @@ wd_status_t host_allreduce(wd_table* t, uint64_t* v, int op) {
 }
 
 // ------------------------------------------------------------------ join helpers
-// make the shard's internal streams wait for `stream`
-wd_status_t fork_from(wd_table* t, cudaStream_t stream, cudaEvent_t* ev_tmp) {
-  CK(cudaEventCreateWithFlags(ev_tmp, cudaEventDisableTiming));
-  CK(cudaEventRecord(*ev_tmp, stream));
-  for (auto& s : t->local) {
+// make the shard's internal streams wait for `stream` (per != nullptr: shard r waits for
+// per[r], the _sharded calls)
+wd_status_t fork_from(wd_table* t, cudaStream_t stream, cudaEvent_t* ev_tmp,
+                      const cudaStream_t* per = nullptr) {
+  *ev_tmp = nullptr;
+  if (!per) {
+    CK(cudaEventCreateWithFlags(ev_tmp, cudaEventDisableTiming));
+    CK(cudaEventRecord(*ev_tmp, stream));
+  }
+  for (size_t r = 0; r < t->local.size(); ++r) {
+    Shard& s = t->local[r];
     DeviceGuard g(s.device);
-    CK(cudaStreamWaitEvent(s.s_main, *ev_tmp, 0));
-    if (s.s_probe != s.s_main) CK(cudaStreamWaitEvent(s.s_probe, *ev_tmp, 0));
-    CK(cudaStreamWaitEvent(s.s_h2d, *ev_tmp, 0));
-    CK(cudaStreamWaitEvent(s.s_d2h, *ev_tmp, 0));
+    cudaEvent_t ev = *ev_tmp;
+    if (per) {
+      CK(cudaEventRecord(s.ev_fork, per[r]));
+      ev = s.ev_fork;
+    }
+    CK(cudaStreamWaitEvent(s.s_main, ev, 0));
+    if (s.s_probe != s.s_main) CK(cudaStreamWaitEvent(s.s_probe, ev, 0));
+    CK(cudaStreamWaitEvent(s.s_h2d, ev, 0));
+    CK(cudaStreamWaitEvent(s.s_d2h, ev, 0));
   }
   return WD_OK;
 }
-// make `stream` wait for all internal streams
-wd_status_t join_into(wd_table* t, cudaStream_t stream, cudaEvent_t ev_tmp) {
-  for (auto& s : t->local) {
+// make `stream` (or per[r] for shard r) wait for all internal streams
+wd_status_t join_into(wd_table* t, cudaStream_t stream, cudaEvent_t ev_tmp,
+                      const cudaStream_t* per = nullptr) {
+  for (size_t r = 0; r < t->local.size(); ++r) {
+    Shard& s = t->local[r];
     DeviceGuard g(s.device);
+    const cudaStream_t out = per ? per[r] : stream;
     CK(cudaEventRecord(s.ev_join_main, s.s_main));
     if (s.s_probe != s.s_main) {
       CK(cudaEventRecord(s.ev_join_probe, s.s_probe));
-      CK(cudaStreamWaitEvent(stream, s.ev_join_probe, 0));
+      CK(cudaStreamWaitEvent(out, s.ev_join_probe, 0));
     }
     CK(cudaEventRecord(s.ev_join_h2d, s.s_h2d));
     CK(cudaEventRecord(s.ev_join_d2h, s.s_d2h));
-    CK(cudaStreamWaitEvent(stream, s.ev_join_main, 0));
-    CK(cudaStreamWaitEvent(stream, s.ev_join_h2d, 0));
-    CK(cudaStreamWaitEvent(stream, s.ev_join_d2h, 0));
+    CK(cudaStreamWaitEvent(out, s.ev_join_main, 0));
+    CK(cudaStreamWaitEvent(out, s.ev_join_h2d, 0));
+    CK(cudaStreamWaitEvent(out, s.ev_join_d2h, 0));
   }
   if (ev_tmp) cudaEventDestroy(ev_tmp);
   return WD_OK;
@@ -567,7 +583,8 @@ wd_status_t agree_batches(wd_table* t, uint64_t local_nbt, uint64_t* global_nbt)
   return WD_OK;
 }
 
-wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t stream) {
+wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t stream,
+                       const cudaStream_t* per = nullptr) {
   const bool insert = op == OP_INSERT;
   TRY(ensure_exchange(t));
   const uint64_t B = t->xbatch;   // a power of two (xchg_batch)
@@ -583,7 +600,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
   TRY(agree_batches(t, local_nbt, &nbt));
   if (nbt == 0) return WD_OK;
   cudaEvent_t ev0;
-  TRY(fork_from(t, stream, &ev0));
+  TRY(fork_from(t, stream, &ev0, per));
 
   // Three phases per batch b (epoch e = epoch0 + 1 + b, exchange slot e % 2):
   //   A (s_main):  multisplit fused with the push into the owners' receive regions, then
@@ -699,7 +716,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
     if (!insert) TRY(phaseC(b));
   }
   t->epoch += nbt;
-  return join_into(t, stream, ev0);
+  return join_into(t, stream, ev0, per);
 }
 
 // split a host/device array over the local shards ("split into portions of
@@ -717,56 +734,67 @@ void split_io(wd_table* t, const IO& all, std::vector<IO>& ios) {
   }
 }
 
-wd_status_t check_ptr(wd_table* t, const void* p, PtrKind* kind) {
+// shard < 0: a whole-table call (device memory only for single-device tables); else the
+// pointer of local shard `shard` in a _sharded call (device memory on that shard's device)
+wd_status_t check_ptr(wd_table* t, const void* p, PtrKind* kind, int shard = -1) {
   int dev = -1;
   *kind = classify(p, &dev);
   if (*kind == PK_DEVICE && p) {
-    if (t->mode == MODE_MULTI)
+    if (shard < 0 && t->mode == MODE_MULTI)
       return fail(WD_ERR_INVALID_ARG,
-                  "device pointers with n_gpus > 1 in one process: pass host memory");
-    if (dev != t->local[0].device)
-      return fail(WD_ERR_INVALID_ARG, "device pointer on device %d, table on device %d", dev,
-                  t->local[0].device);
+                  "device pointers with n_gpus > 1 in one process: pass host memory or use "
+                  "wd_insert_sharded / wd_retrieve_sharded");
+    const int want = t->local[shard < 0 ? 0 : shard].device;
+    if (dev != want)
+      return fail(WD_ERR_INVALID_ARG, "device pointer on device %d, shard on device %d", dev, want);
   }
   return WD_OK;
 }
 
-wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* vals,
-                  uint32_t* vout, uint8_t* fout, uint64_t n, cudaStream_t stream) {
-  const bool insert = op == OP_INSERT;
-  if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
-  if (n && !keys) return fail(WD_ERR_INVALID_ARG, "keys == NULL with n > 0");
-  if (n && insert && !vals) return fail(WD_ERR_INVALID_ARG, "vals == NULL with n > 0");
-  IO io;
-  io.keys = keys; io.vals = vals; io.vout = vout; io.fout = fout; io.n = n;
-  if (n) {
-    PtrKind k1, k2 = PK_DEVICE, k3 = PK_DEVICE;
-    TRY(check_ptr(t, keys, &k1));
-    if (insert) TRY(check_ptr(t, vals, &k2));
-    else {
-      if (vout) TRY(check_ptr(t, vout, &k2));
-      if (fout) TRY(check_ptr(t, fout, &k3));
-    }
-    if (insert && (k1 == PK_DEVICE) != (k2 == PK_DEVICE))
-      return fail(WD_ERR_INVALID_ARG, "keys and vals must both be host or both device");
-    if (!insert && vout && fout && (k2 == PK_DEVICE) != (k3 == PK_DEVICE))
-      return fail(WD_ERR_INVALID_ARG, "vals_out and found_out must both be host or device");
-    io.kin = (k1 == PK_PAGEABLE || k2 == PK_PAGEABLE) && insert ? PK_PAGEABLE : k1;
-    io.kout = insert ? PK_DEVICE : (vout ? k2 : k3);
-    if (!insert && !vout && !fout) io.kout = PK_DEVICE;
+// pointer kinds of one call's buffers (same rules for whole-table and per-shard calls)
+wd_status_t classify_io(wd_table* t, bool insert, IO& io, int shard) {
+  if (!io.n) return WD_OK;
+  if (!io.keys) return fail(WD_ERR_INVALID_ARG, "keys == NULL with n > 0");
+  if (insert && !io.vals) return fail(WD_ERR_INVALID_ARG, "vals == NULL with n > 0");
+  PtrKind k1, k2 = PK_DEVICE, k3 = PK_DEVICE;
+  TRY(check_ptr(t, io.keys, &k1, shard));
+  if (insert) TRY(check_ptr(t, io.vals, &k2, shard));
+  else {
+    if (io.vout) TRY(check_ptr(t, io.vout, &k2, shard));
+    if (io.fout) TRY(check_ptr(t, io.fout, &k3, shard));
   }
-  // P:245 future work, built: "a heuristic which dynamically scales the group size |g|
-  // with the current load factor".  P:89 makes switching |g| between calls safe (same probe
-  // sequence).  Measured on B200 (profiles/r01_sweep.jsonl, 2^28 keys, insert + retrieve
-  // step): |g| = 8 is fastest up to alpha 0.9, |g| = 16 from 0.95 on (and for misses at any
-  // load).  The load used is the projected one after this call, from a host-side upper
-  // estimate of the size (no synchronisation).
+  if (insert && (k1 == PK_DEVICE) != (k2 == PK_DEVICE))
+    return fail(WD_ERR_INVALID_ARG, "keys and vals must both be host or both device");
+  if (!insert && io.vout && io.fout && (k2 == PK_DEVICE) != (k3 == PK_DEVICE))
+    return fail(WD_ERR_INVALID_ARG, "vals_out and found_out must both be host or device");
+  io.kin = (k1 == PK_PAGEABLE || k2 == PK_PAGEABLE) && insert ? PK_PAGEABLE : k1;
+  io.kout = insert ? PK_DEVICE : (io.vout ? k2 : k3);
+  if (!insert && !io.vout && !io.fout) io.kout = PK_DEVICE;
+  return WD_OK;
+}
+
+// P:245 future work, built: "a heuristic which dynamically scales the group size |g| with
+// the current load factor".  P:89 makes switching |g| between calls safe (same probe
+// sequence).  Measured on B200 (profiles/r01_sweep.jsonl, 2^28 keys, insert + retrieve
+// step): |g| = 8 is fastest up to alpha 0.9, |g| = 16 from 0.95 on (and for misses at any
+// load).  The load used is the projected one after this call, from a host-side upper
+// estimate of the size (no synchronisation).
+void pick_group_size(wd_table* t, int op, uint64_t n) {
   if (t->G == 0) {
     const double cap = double(wd_capacity(t));
     const double est = double(t->est_size) + (op == OP_INSERT ? double(n) : 0.0);
     t->G_used = (est / cap > 0.93) ? 16 : 8;
   }
   if (op == OP_INSERT) t->est_size = std::min<uint64_t>(t->est_size + n, wd_capacity(t));
+}
+
+wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* vals,
+                  uint32_t* vout, uint8_t* fout, uint64_t n, cudaStream_t stream) {
+  if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  IO io;
+  io.keys = keys; io.vals = vals; io.vout = vout; io.fout = fout; io.n = n;
+  TRY(classify_io(t, op == OP_INSERT, io, -1));
+  pick_group_size(t, op, n);
   if (t->m == 1) {
     if (n == 0) return WD_OK;
     return single_op(t, op, io, stream);
@@ -774,6 +802,37 @@ wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* val
   std::vector<IO> ios;
   split_io(t, io, ios);
   return cascade_op(t, op, ios, stream);
+}
+
+// The paper's device-sided cascades: every local shard brings its own
+// device-resident portion ("split into portions"), on its own stream.
+wd_status_t do_op_sharded(wd_table* t, int op, const uint32_t* const* keys,
+                          const uint32_t* const* vals, uint32_t* const* vout, uint8_t* const* fout,
+                          const uint64_t* n, const wd_stream_t* streams) {
+  if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  if (!keys || !n || (op == OP_INSERT && !vals))
+    return fail(WD_ERR_INVALID_ARG, "_sharded: NULL array argument");
+  const size_t L = t->local.size();
+  std::vector<IO> ios(L);
+  std::vector<cudaStream_t> per(L, nullptr);
+  uint64_t total = 0;
+  for (size_t r = 0; r < L; ++r) {
+    IO& io = ios[r];
+    io.keys = keys[r];
+    io.vals = vals ? vals[r] : nullptr;
+    io.vout = vout ? vout[r] : nullptr;
+    io.fout = fout ? fout[r] : nullptr;
+    io.n = n[r];
+    if (streams) per[r] = reinterpret_cast<cudaStream_t>(streams[r]);
+    TRY(classify_io(t, op == OP_INSERT, io, int(r)));
+    total += n[r];
+  }
+  pick_group_size(t, op, total);
+  if (t->m == 1) {
+    if (ios[0].n == 0) return WD_OK;
+    return single_op(t, op, ios[0], per[0]);
+  }
+  return cascade_op(t, op, ios, nullptr, per.data());
 }
 
 wd_table* create_common(uint64_t capacity, int mode, int m, int group_size) {
@@ -1034,6 +1093,17 @@ wd_status_t wd_retrieve(wd_table_t* t, const uint32_t* keys, uint32_t* vals_out,
                         uint64_t n, wd_stream_t stream) {
   return do_op(t, OP_RETRIEVE, keys, nullptr, vals_out, found_out, n,
                reinterpret_cast<cudaStream_t>(stream));
+}
+
+wd_status_t wd_insert_sharded(wd_table_t* t, const uint32_t* const keys[], const uint32_t* const vals[],
+                              const uint64_t n[], const wd_stream_t streams[]) {
+  return do_op_sharded(t, OP_INSERT, keys, vals, nullptr, nullptr, n, streams);
+}
+
+wd_status_t wd_retrieve_sharded(wd_table_t* t, const uint32_t* const keys[], uint32_t* const vals_out[],
+                                uint8_t* const found_out[], const uint64_t n[],
+                                const wd_stream_t streams[]) {
+  return do_op_sharded(t, OP_RETRIEVE, keys, nullptr, vals_out, found_out, n, streams);
 }
 
 wd_status_t wd_erase(wd_table_t* t, const uint32_t* keys, uint8_t* found_out, uint64_t n,

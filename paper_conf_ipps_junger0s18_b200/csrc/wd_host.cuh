@@ -106,6 +106,7 @@ struct Shard {
   cudaEvent_t ev_h2d[kStage] = {}, ev_free[kStage] = {}, ev_kdone[kStage] = {}, ev_d2h[kStage] = {};
   cudaEvent_t ev_join_main = nullptr, ev_join_h2d = nullptr, ev_join_d2h = nullptr;
   cudaEvent_t ev_join_probe = nullptr;
+  cudaEvent_t ev_fork = nullptr;   // _sharded calls: this shard's caller stream
   bool h2d_pending[kStage] = {};   // the slot's staging buffers have a pending release (ev_free)
   bool l2_held = false;            // holds the device's L2 fetch-granularity setting
 };

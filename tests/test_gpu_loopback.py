@@ -110,3 +110,37 @@ def test_loopback_zipf(wd, m):
     mo.insert(keys, vals)
     assert np.all(gf == 1)
     assert np.all(mo.pair_status(q, gv) >= 1)
+
+
+@pytest.mark.parametrize("m", [2, 4])
+def test_loopback_sharded_calls(wd, m):
+    # wd_insert_sharded / wd_retrieve_sharded (the device-sided cascade of
+    # P:175 / P:199): every shard brings its own device-resident portion on its own stream;
+    # every query of every portion against the closed form
+    import torch
+    import wdgen.gpu as gg
+    n_local, ks, vs = 150_001, 91, 92
+    n = n_local * m
+    with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=m) as t:
+        t.set_option(wd.WD_OPT_BATCH, 40_000)
+        assert t.get_option(wd.WD_OPT_LOCAL_SHARDS) == m
+        keys = [gg.unique_keys(n_local, ks, start=r * n_local) for r in range(m)]
+        vals = [gg.values(n_local, vs, start=r * n_local) for r in range(m)]
+        streams = [torch.cuda.Stream() for _ in range(m)]
+        for s in streams:                        # the portions were generated on this stream
+            s.wait_stream(torch.cuda.current_stream())
+        t.insert_sharded(keys, vals, streams)
+        q = [gg.interleaved_queries(n, ks, start=r * 2 * n_local, count=2 * n_local) for r in range(m)]
+        vo = [torch.empty(2 * n_local, dtype=torch.int32, device="cuda") for _ in range(m)]
+        fo = [torch.empty(2 * n_local, dtype=torch.uint8, device="cuda") for _ in range(m)]
+        for s in streams:
+            s.wait_stream(torch.cuda.current_stream())
+        t.retrieve_sharded(q, vo, fo, streams)
+        torch.cuda.synchronize()
+        assert t.sync() == 0 and t.size() == n
+        for r in range(m):
+            bad, first, found = gg.check_unique(q[r], vo[r], fo[r], n, ks, vs)
+            assert bad == 0, (r, bad, first)
+            assert found == n_local
+        with pytest.raises(ValueError):
+            t.insert_sharded(keys[:1], vals[:1])

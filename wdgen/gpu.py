@@ -20,6 +20,7 @@ def lib():
         L.wdgen_interleaved_queries.argtypes = [p, u64, u64, u64, u64, p]
         L.wdgen_mixed_queries.argtypes = [p, p, u64, u64, u64, C.c_double, u64, p]
         L.wdgen_zipf_keys.argtypes = [p, u64, u64, u64, u64, p]
+        L.wdgen_check_unique.argtypes = [p, p, p, u64, u64, u64, u64, p, p]
         _lib = L
     return _lib
 
@@ -77,3 +78,27 @@ def zipf_keys(n, universe, seed, start=0, out=None):
     out = _new(n) if out is None else out
     _chk(lib().wdgen_zipf_keys(out.data_ptr(), start, n, universe, seed, _s()))
     return out
+
+
+def check_unique(q, vals_out, found_out, n_present, key_seed, val_seed, chunk=1 << 28):
+    """Closed-form check of EVERY query on the device (test harness): query k must report
+    found iff pi_s^-1(k) < n_present, with value values(pi_s^-1(k)) (else WD_NOT_FOUND).
+    vals_out / found_out may be None.  Returns (mismatches, first mismatching position or
+    None, found count).  Generator arithmetic only (wdgen), no code of the method."""
+    import torch
+    res = torch.tensor([0, -1, 0], dtype=torch.int64, device=q.device)
+    n = q.numel()
+    for o in range(0, n, chunk):
+        c = min(chunk, n - o)
+        r = torch.tensor([0, -1, 0], dtype=torch.int64, device=q.device)
+        vp = vals_out[o:o + c].data_ptr() if vals_out is not None else None
+        fp = found_out[o:o + c].data_ptr() if found_out is not None else None
+        _chk(lib().wdgen_check_unique(q[o:o + c].data_ptr(), vp, fp, c, n_present, key_seed,
+                                      val_seed, r.data_ptr(), _s()))
+        bad, first, found = r.tolist()
+        res[0] += bad
+        res[2] += found
+        if bad and res[1].item() == -1:
+            res[1] = o + first
+    bad, first, found = res.tolist()
+    return int(bad), (int(first) if bad else None), int(found)

@@ -80,6 +80,63 @@ __global__ void k_mixed(uint32_t* out, uint8_t* hit_out, uint64_t n_table, uint6
     if (hit_out) hit_out[i] = hit;
   }
 }
+// ---- closed-form checker (test harness; generator arithmetic only, none of the method's):
+// a key k is present iff its generator index pi_s^-1(k) < n_present, and then its value is
+// values(pi_s^-1(k)) — the same closed form as oracle.expected_unique, evaluated on the
+// device so full-size runs can check EVERY query.  res[0] += mismatches, res[1] = min
+// mismatching position, res[2] += found count.
+__device__ inline uint32_t feistel_inv(uint32_t y, const RK& rk) {
+  uint64_t L = y >> 16, R = y & 0xFFFF;
+#pragma unroll
+  for (int r = 3; r >= 0; --r) {
+    const uint64_t F = splitmix64(L ^ rk.k[r]) & 0xFFFF;
+    const uint64_t nl = R ^ F;
+    R = L;
+    L = nl;
+  }
+  return uint32_t((L << 16) | R);
+}
+__device__ inline uint32_t perm32_inv(uint32_t y, const RK& rk) {
+  uint32_t x = feistel_inv(y, rk);
+  if (x == kEmpty) x = feistel_inv(kEmpty, rk);
+  return x;
+}
+__global__ void k_check_unique(const uint32_t* q, const uint32_t* vout, const uint8_t* fout,
+                               uint64_t count, uint64_t n_present, uint64_t vsk, RK rk,
+                               unsigned long long* res) {
+  unsigned long long bad = 0, found = 0, first = ~0ull;
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < count; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t k = q[i];
+    bool present = false;
+    uint32_t ev = 0xFFFFFFFFu;
+    if (k != kEmpty) {
+      const uint64_t idx = perm32_inv(k, rk);
+      present = idx < n_present;
+      if (present) ev = uint32_t(splitmix64(idx + vsk));
+    }
+    bool ok = true;
+    if (fout) {
+      ok = ok && (fout[i] == (present ? 1 : 0));
+      found += fout[i] == 1;
+    }
+    if (vout) ok = ok && vout[i] == ev;
+    if (!ok) {
+      ++bad;
+      if (i < first) first = i;
+    }
+  }
+  for (int o = 16; o; o >>= 1) {
+    bad += __shfl_xor_sync(0xFFFFFFFFu, bad, o);
+    found += __shfl_xor_sync(0xFFFFFFFFu, found, o);
+    const unsigned long long f2 = __shfl_xor_sync(0xFFFFFFFFu, first, o);
+    first = f2 < first ? f2 : first;
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (bad) { atomicAdd(res, bad); atomicMin(res + 1, first); }
+    if (found) atomicAdd(res + 2, found);
+  }
+}
+
 // exact Zipf by rejection-inversion — the same computation as wdgen.zipf_ranks
 struct ZipfC { double expo, c1, cn, sq, universe; };
 __host__ __device__ inline double zh1(double x) {
@@ -154,6 +211,14 @@ int wdgen_zipf_keys(uint32_t* out, uint64_t start, uint64_t n, uint64_t universe
                     cudaStream_t st) {
   if (n) k_zipf<<<grid_for(n), 256, 0, st>>>(out, start, n, stream_key(seed, TAG_ZIPF),
                                              zipf_consts(universe, 1.0 + 1e-6), round_keys(seed));
+  return int(cudaGetLastError());
+}
+int wdgen_check_unique(const uint32_t* q, const uint32_t* vout, const uint8_t* fout, uint64_t count,
+                       uint64_t n_present, uint64_t key_seed, uint64_t val_seed,
+                       unsigned long long* res, cudaStream_t st) {
+  if (count)
+    k_check_unique<<<grid_for(count), 256, 0, st>>>(q, vout, fout, count, n_present,
+                                                    stream_key(val_seed, TAG_VAL), round_keys(key_seed), res);
   return int(cudaGetLastError());
 }
 int wdgen_mixed_queries(uint32_t* out, uint8_t* hit_out, uint64_t n_table, uint64_t start, uint64_t count,
