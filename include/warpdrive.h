@@ -48,7 +48,8 @@ typedef enum {
     WD_ERR_INVALID_ARG = 1,
     WD_ERR_OUT_OF_MEMORY = 2,
     WD_ERR_CUDA = 3,
-    WD_ERR_NCCL = 4,           /* reserved (the exchange does not use NCCL) */
+    WD_ERR_NCCL = 4,           /* NCCL exchange (WD_OPT_EXCHANGE = 2): NCCL not loadable or an
+                                  NCCL call failed (text: wd_last_error_message) */
     WD_ERR_TABLE_FULL = 5,     /* >=1 insert exhausted p_max regions (Fig. 3 Line 26);
                                   that pair was dropped */
     WD_ERR_RESERVED_KEY = 6,   /* >=1 input key == WD_EMPTY_KEY; those pairs were skipped
@@ -97,7 +98,7 @@ wd_table_t* wd_create_loopback(uint64_t capacity, int n_shards, int group_size);
  * place, returns 0 on success); it is called synchronously, in the same order on every
  * rank, for control only (batch-count agreement, wd_size, barriers) — the data path is
  * peer-memory stores/loads inside the kernels.  WD_OPT_BATCH is fixed once connected. */
-#define WD_RANK_HANDLE_BYTES 128
+#define WD_RANK_HANDLE_BYTES 256
 #define WD_REDUCE_SUM 0
 #define WD_REDUCE_MAX 1
 typedef int (*wd_allreduce_fn)(uint64_t* value, int op, void* ctx);
@@ -224,6 +225,24 @@ typedef enum {
                                 at most 2^26 pairs at a time, kept for the table's lifetime
                                 (stream-ordered allocation); in auto mode a failed scratch
                                 allocation falls back to the plain launch. */
+    WD_OPT_EXCHANGE = 12,    /* how the transposition of P:117 (a8) and its reverse (a10) move
+                                data between shards (m > 1):
+                                0 (default): fused — the multisplit kernel stores every item
+                                  straight into its owner's receive region and the owner's
+                                  probe kernel stores every answer straight into its origin's
+                                  result region (peer memory over NVLink, epoch flags, no
+                                  host synchronisation);
+                                1: staged + copy engine — local per-destination send buckets,
+                                  then one cudaMemcpyAsync of the exact count per peer (the
+                                  paper's asynchronous inter-GPU copies), results back
+                                  the same way; the host reads its row of T per batch;
+                                2: staged + NCCL — T all-gathered with ncclAllGather, then an
+                                  all-to-all(v) of the exact counts as grouped ncclSend /
+                                  ncclRecv (forward and reverse on two communicators).  Needs
+                                  one GPU per shard (wd_create with n_gpus > 1, or rank mode;
+                                  rank mode: set before wd_rank_handle).  NCCL is loaded at
+                                  run time (libnccl.so.2).
+                                Results are identical in all three modes. */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -31,10 +31,12 @@ WD_NOT_FOUND = 0xFFFFFFFF
 WD_OPT_GROUP_SIZE, WD_OPT_P_MAX, WD_OPT_BATCH, WD_OPT_SERIAL = 0, 1, 2, 3
 WD_OPT_KEYS_IN_FLIGHT, WD_OPT_PART_SEED, WD_OPT_PART_MODE, WD_OPT_PROBE_MODE = 4, 5, 6, 7
 WD_OPT_KERNEL_FLAGS, WD_OPT_SLOTS_PER_LANE, WD_OPT_SPAN, WD_OPT_SLICES = 8, 9, 10, 11
+WD_OPT_EXCHANGE = 12
+EXCHANGE_FUSED, EXCHANGE_COPY, EXCHANGE_NCCL = 0, 1, 2
 WD_OPT_N_SHARDS, WD_OPT_RANK, WD_OPT_LOCAL_SHARDS, WD_OPT_LAUNCHES = 100, 101, 102, 103
 WD_OPT_GROUP_SIZE_USED = 104
 WD_OPT_REGION_ALIGN = 105
-WD_RANK_HANDLE_BYTES = 128
+WD_RANK_HANDLE_BYTES = 256
 # int (*)(uint64_t* value, int op, void* ctx)
 ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.POINTER(C.c_uint64), C.c_int, C.c_void_p)
 
@@ -155,7 +157,8 @@ class Table:
 
     def __init__(self, capacity: int, n_gpus: int = 1, group_size: int = 4, *,
                  loopback_shards: int | None = None, rank: int | None = None,
-                 world: int | None = None, process_group=None, batch: int | None = None):
+                 world: int | None = None, process_group=None, batch: int | None = None,
+                 exchange: int | None = None):
         """rank/world: one process per GPU (torchrun); the exchange handles are all-gathered
         and the host collective is run over `process_group` (torch.distributed)."""
         self._cb = None
@@ -171,6 +174,8 @@ class Table:
         self._h = h
         if batch is not None:
             self.set_option(WD_OPT_BATCH, batch)
+        if exchange is not None:        # rank mode: before the handles are exchanged
+            self.set_option(WD_OPT_EXCHANGE, exchange)
         if rank is not None:
             self._connect(process_group)
 

@@ -17,6 +17,8 @@
 // =====================================================================================
 #include "wd_host.cuh"
 
+#include <dlfcn.h>
+
 #include <mutex>
 
 namespace wdi {
@@ -32,6 +34,69 @@ wd_status_t fail(wd_status_t s, const char* fmt, ...) {
   g_last = s;
   return s;
 }
+
+// ------------------------------------------------------------------ NCCL (WD_OPT_EXCHANGE = 2)
+// Loaded at run time (dlopen), so the library needs NCCL only when the NCCL exchange is
+// selected: the copy already in the process (torch's), else libnccl.so.2 from the loader
+// path.  Only ABI-stable NCCL 2.x types are used (ncclUniqueId = 128 bytes, ncclUint8 = 1,
+// ncclUint64 = 5).
+struct NcclUid { char internal[128]; };
+constexpr int kNcclUint8 = 1, kNcclUint64 = 5;
+struct NcclApi {
+  bool tried = false, ok = false;
+  char why[256] = "";
+  int (*GetUniqueId)(NcclUid*) = nullptr;
+  int (*CommInitRank)(void**, int, NcclUid, int) = nullptr;
+  int (*CommInitAll)(void**, int, const int*) = nullptr;
+  int (*CommSplit)(void*, int, int, void**, void*) = nullptr;
+  int (*CommDestroy)(void*) = nullptr;
+  int (*GroupStart)() = nullptr;
+  int (*GroupEnd)() = nullptr;
+  int (*Send)(const void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  int (*Recv)(void*, size_t, int, int, void*, cudaStream_t) = nullptr;
+  int (*AllGather)(const void*, void*, size_t, int, void*, cudaStream_t) = nullptr;
+  const char* (*GetErrorString)(int) = nullptr;
+};
+NcclApi g_nccl;
+std::mutex g_nccl_mu;
+
+const NcclApi* nccl_api() {
+  std::lock_guard<std::mutex> lk(g_nccl_mu);
+  NcclApi& a = g_nccl;
+  if (a.tried) return a.ok ? &a : nullptr;
+  a.tried = true;
+  void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+  if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+  if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+  if (!h) {
+    snprintf(a.why, sizeof a.why, "libnccl.so.2 not loadable: %s", dlerror());
+    return nullptr;
+  }
+#define WD_NCCL_SYM(f, name)                                                        \
+  a.f = reinterpret_cast<decltype(a.f)>(dlsym(h, name));                            \
+  if (!a.f) { snprintf(a.why, sizeof a.why, "NCCL symbol %s missing", name); return nullptr; }
+  WD_NCCL_SYM(GetUniqueId, "ncclGetUniqueId")
+  WD_NCCL_SYM(CommInitRank, "ncclCommInitRank")
+  WD_NCCL_SYM(CommInitAll, "ncclCommInitAll")
+  WD_NCCL_SYM(CommSplit, "ncclCommSplit")
+  WD_NCCL_SYM(CommDestroy, "ncclCommDestroy")
+  WD_NCCL_SYM(GroupStart, "ncclGroupStart")
+  WD_NCCL_SYM(GroupEnd, "ncclGroupEnd")
+  WD_NCCL_SYM(Send, "ncclSend")
+  WD_NCCL_SYM(Recv, "ncclRecv")
+  WD_NCCL_SYM(AllGather, "ncclAllGather")
+  WD_NCCL_SYM(GetErrorString, "ncclGetErrorString")
+#undef WD_NCCL_SYM
+  a.ok = true;
+  return &a;
+}
+#define NK(x)                                                                              \
+  do {                                                                                     \
+    const int r_ = (x);                                                                    \
+    if (r_ != 0)                                                                           \
+      return fail(WD_ERR_NCCL, "%s: %s (%s:%d)", #x, g_nccl.GetErrorString(r_), __FILE__, \
+                  __LINE__);                                                               \
+  } while (0)
 
 // ------------------------------------------------------------------ L2 fetch granularity
 // Random 32-byte windows: do not let L2 promote a sector miss to a 64/128-byte DRAM fetch
@@ -283,10 +348,12 @@ struct RankHandle {
   char ipc[64];
   uint64_t magic, batch, arena_bytes;
   uint32_t world, rank;
-  char pad[WD_RANK_HANDLE_BYTES - 64 - 3 * 8 - 2 * 4];
+  uint32_t exchange, has_nccl_id;       // rank 0: an ncclUniqueId follows (WD_OPT_EXCHANGE = 2)
+  char nccl_id[128];
+  char pad[WD_RANK_HANDLE_BYTES - 64 - 3 * 8 - 4 * 4 - 128];
 };
 static_assert(sizeof(RankHandle) == WD_RANK_HANDLE_BYTES, "rank handle size");
-constexpr uint64_t kHandleMagic = 0x5744524B48444C31ull;  // "WDRKHDL1"
+constexpr uint64_t kHandleMagic = 0x5744524B48444C32ull;  // "WDRKHDL2"
 
 wd_status_t host_allreduce(wd_table* t, uint64_t* v, int op) {
   if (t->mode != MODE_RANK) return WD_OK;
@@ -583,35 +650,167 @@ wd_status_t agree_batches(wd_table* t, uint64_t local_nbt, uint64_t* global_nbt)
   return WD_OK;
 }
 
+// ------------------------------------------------------------------ staged exchange
+void free_staged(Shard& s) {
+  DeviceGuard g(s.device);
+  if (s.send) cudaFree(s.send);
+  if (s.res_stage) cudaFree(s.res_stage);
+  s.send = nullptr;
+  s.res_stage = nullptr;
+  for (int i = 0; i < 2; ++i) {
+    if (s.hrow[i]) cudaFreeHost(s.hrow[i]);
+    if (s.hcol[i]) cudaFreeHost(s.hcol[i]);
+    if (s.hT[i]) cudaFreeHost(s.hT[i]);
+    if (s.Tdev[i]) cudaFree(s.Tdev[i]);
+    s.hrow[i] = s.hcol[i] = s.hT[i] = s.Tdev[i] = nullptr;
+    for (cudaEvent_t* e : {&s.ev_ready[i], &s.ev_pdone[i], &s.ev_done[i], &s.ev_unperm[i]}) {
+      if (*e) cudaEventDestroy(*e);
+      *e = nullptr;
+    }
+    s.pdone_rec[i] = s.unperm_rec[i] = false;
+  }
+  if (s.ev_row) cudaEventDestroy(s.ev_row);
+  if (s.ev_col) cudaEventDestroy(s.ev_col);
+  s.ev_row = s.ev_col = nullptr;
+  s.staged_B = 0;
+}
+
+void free_nccl(wd_table* t) {
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    if (s.comm_rev) g_nccl.CommDestroy(s.comm_rev);
+    if (s.comm_fwd) g_nccl.CommDestroy(s.comm_fwd);
+    s.comm_fwd = s.comm_rev = nullptr;
+  }
+  t->nccl_ready = false;
+}
+
+// the staged transport's buffers for batch size B: send [m][B] items (u64 pairs or u32 keys),
+// res_stage [m][B] packed results, pinned rows / columns of T per exchange slot
+wd_status_t ensure_staged(wd_table* t, Shard& s, uint64_t B) {
+  if (s.staged_B == B) return WD_OK;
+  free_staged(s);
+  DeviceGuard g(s.device);
+  const int m = t->m;
+  CK(cudaMalloc(&s.send, size_t(m) * B * 8));
+  CK(cudaMalloc(&s.res_stage, size_t(m) * B * 8));
+  for (int i = 0; i < 2; ++i) {
+    CK(cudaMallocHost(&s.hrow[i], m * 8));
+    CK(cudaMallocHost(&s.hcol[i], m * 8));
+    CK(cudaMallocHost(&s.hT[i], size_t(m) * m * 8));
+    CK(cudaMalloc(&s.Tdev[i], size_t(m) * m * 8));
+    for (cudaEvent_t* e : {&s.ev_ready[i], &s.ev_pdone[i], &s.ev_done[i], &s.ev_unperm[i]})
+      CK(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+  }
+  CK(cudaEventCreateWithFlags(&s.ev_row, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&s.ev_col, cudaEventDisableTiming));
+  s.staged_B = B;
+  return WD_OK;
+}
+
+// NCCL communicators of the forward and the reverse transposition (collective: every rank
+// calls it at its first NCCL-exchange operation, in the same order)
+wd_status_t ensure_nccl(wd_table* t) {
+  if (t->nccl_ready) return WD_OK;
+  const NcclApi* a = nccl_api();
+  if (!a) return fail(WD_ERR_NCCL, "%s", g_nccl.why);
+  if (t->mode == MODE_MULTI) {
+    std::vector<void*> c(t->m, nullptr);
+    std::vector<int> devs(t->m);
+    for (int r = 0; r < t->m; ++r) devs[r] = t->local[r].device;
+    NK(a->CommInitAll(c.data(), t->m, devs.data()));
+    for (int r = 0; r < t->m; ++r) t->local[r].comm_fwd = c[r];
+    NK(a->CommInitAll(c.data(), t->m, devs.data()));
+    for (int r = 0; r < t->m; ++r) t->local[r].comm_rev = c[r];
+  } else if (t->mode == MODE_RANK) {
+    if (!t->have_nccl_id)
+      return fail(WD_ERR_NCCL, "rank mode: set WD_OPT_EXCHANGE = 2 before wd_rank_handle / "
+                               "wd_rank_connect (rank 0's NCCL id travels in the handles)");
+    Shard& s = t->local[0];
+    DeviceGuard g(s.device);
+    NcclUid id;
+    memcpy(&id, t->nccl_id, sizeof id);
+    NK(a->CommInitRank(&s.comm_fwd, t->m, id, t->rank));
+    NK(a->CommSplit(s.comm_fwd, 0, t->rank, &s.comm_rev, nullptr));
+  } else {
+    return fail(WD_ERR_UNSUPPORTED, "the NCCL exchange needs one GPU per shard (wd_create with "
+                                    "n_gpus > 1, or rank mode); loopback shards share a device");
+  }
+  t->nccl_ready = true;
+  return WD_OK;
+}
+
 wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t stream,
                        const cudaStream_t* per = nullptr) {
   const bool insert = op == OP_INSERT;
   TRY(ensure_exchange(t));
   const uint64_t B = t->xbatch;   // a power of two (xchg_batch)
   const int m = t->m;
+  const int X = t->exchange;      // 0 fused, 1 staged + copy engine, 2 staged + NCCL
+  if (X == 2) TRY(ensure_nccl(t));
   uint64_t local_nbt = 0;
   for (size_t r = 0; r < t->local.size(); ++r) {
     local_nbt = std::max(local_nbt, (ios[r].n + B - 1) / B);
     if (needs_staging(ios[r]))
       TRY(ensure_staging(t->local[r], B,
                          ios[r].kin == PK_PAGEABLE || ios[r].kout == PK_PAGEABLE));
+    if (X) TRY(ensure_staged(t, t->local[r], B));
   }
   uint64_t nbt = 0;
   TRY(agree_batches(t, local_nbt, &nbt));
   if (nbt == 0) return WD_OK;
   cudaEvent_t ev0;
   TRY(fork_from(t, stream, &ev0, per));
+  const size_t isz = insert ? 8 : 4;          // bytes per exchanged item (pair / key)
+  const bool all_local = t->mode != MODE_RANK;  // this process holds every row of T
 
   // Three phases per batch b (epoch e = epoch0 + 1 + b, exchange slot e % 2):
-  //   A (s_main):  multisplit fused with the push into the owners' receive regions, then
-  //                publish the row of T and the READY flags
-  //   B (s_probe): wait for the column of T, probe (insert / retrieve), DONE flags
-  //   C (s_main):  queries only — unpermute the results the owners pushed into this shard's
-  //                result slot (local gather), RESC flags (the slot may be reused)
+  //   A (s_main):  multisplit; fused (X = 0): straight into the owners' receive regions,
+  //                then publish the row of T and the READY flags.  Staged (X = 1, 2): into
+  //                the local send buffer, then the transposition proper (phase T below).
+  //   B (s_probe): wait for the column of T, probe (insert / retrieve); queries send their
+  //                results back (fused: peer stores in the probe kernel; staged: res_stage,
+  //                then copy engine / NCCL), DONE flags / events
+  //   C (s_main):  queries only — unpermute the results that arrived in this shard's result
+  //                slot (local gather), RESC flags / events (the slot may be reused)
   // Issued as A(0), then A(b+1), B(b), C(b): the multisplit and transposition of batch b+1
   // overlap the probing of batch b (Fig. 5's MST || INS), and the query's unpermute of
-  // batch b never blocks the next multisplit.  Cross-shard ordering is by epoch flags only.
+  // batch b never blocks the next multisplit.  Fused and copy-engine: cross-shard ordering by
+  // epoch flags only; NCCL: by the collective's own completion, recorded in events.
   const unsigned long long e0 = t->epoch;
+  auto multisplit = [&](Shard& s, const uint32_t* dk, const uint32_t* dv, uint64_t cnt,
+                        int slot) -> wd_status_t {
+    wd::DstPtrs dst{};
+    for (int d = 0; d < m; ++d) {
+      if (X) dst.p[d] = static_cast<char*>(s.send) + uint64_t(d) * B * isz;   // local buckets
+      else if (insert) dst.p[d] = t->peers[d].recv[slot] + uint64_t(s.id) * B;
+      else dst.p[d] = reinterpret_cast<uint32_t*>(t->peers[d].recv[slot]) + uint64_t(s.id) * B;
+    }
+    // every resident block of the SM (occupancy API): more tiles in flight per SM
+    const uint64_t tiles = (cnt + wd::kMsTile - 1) / wd::kMsTile;
+    const int per_sm = insert ? blocks_per_sm(wd::multisplit_kernel<true>)
+                              : blocks_per_sm(wd::multisplit_kernel<false>);
+    const int grid = int(std::min<uint64_t>(tiles, uint64_t(t->sm_count) * per_sm));
+    if (insert)
+      wd::multisplit_kernel<true><<<grid, wd::kBlock, 0, s.s_main>>>(
+          dk, dv, cnt, dst, s.cursor[slot], nullptr, m, t->pseed, t->pmode, B, s.counters);
+    else
+      wd::multisplit_kernel<false><<<grid, wd::kBlock, 0, s.s_main>>>(
+          dk, nullptr, cnt, dst, s.cursor[slot], s.pos[slot], m, t->pseed, t->pmode, B,
+          s.counters);
+    CK(cudaGetLastError());
+    t->launches++;
+    return WD_OK;
+  };
+  auto publish = [&](Shard& s, int slot, unsigned long long e) -> wd_status_t {
+    wd::FlagPtrs cnt_dst{};
+    for (int d = 0; d < m; ++d) cnt_dst.p[d] = t->peers[d].recv_count[slot] + s.id;
+    wd::publish_kernel<<<1, 32, 0, s.s_main>>>(s.cursor[slot], cnt_dst,
+                                               flag_ptrs(t, FLAG_READY, s.id), m, e);
+    CK(cudaGetLastError());
+    t->launches++;
+    return WD_OK;
+  };
   auto phaseA = [&](uint64_t b) -> wd_status_t {
     const unsigned long long e = e0 + 1 + b;
     const int slot = int(e & 1);
@@ -622,35 +821,79 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       const uint64_t off = std::min(io.n, b * B), cnt = std::min(B, io.n - off);
       const uint32_t *dk = nullptr, *dv = nullptr;
       TRY(stage_in(s, io, off, cnt, int(b % kStage), insert, &dk, &dv));
-      if (e > 2) TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e - 2));  // owners released e-2
-      if (cnt) {
-        wd::DstPtrs dst{};
-        for (int d = 0; d < m; ++d) {
-          if (insert) dst.p[d] = t->peers[d].recv[slot] + uint64_t(s.id) * B;
-          else dst.p[d] = reinterpret_cast<uint32_t*>(t->peers[d].recv[slot]) + uint64_t(s.id) * B;
-        }
-        // every resident block of the SM (occupancy API): more tiles in flight per SM
-        const uint64_t tiles = (cnt + wd::kMsTile - 1) / wd::kMsTile;
-        const int per_sm = insert ? blocks_per_sm(wd::multisplit_kernel<true>)
-                                  : blocks_per_sm(wd::multisplit_kernel<false>);
-        const int grid = int(std::min<uint64_t>(tiles, uint64_t(t->sm_count) * per_sm));
-        if (insert)
-          wd::multisplit_kernel<true><<<grid, wd::kBlock, 0, s.s_main>>>(
-              dk, dv, cnt, dst, s.cursor[slot], nullptr, m, t->pseed, t->pmode, B, s.counters);
-        else
-          wd::multisplit_kernel<false><<<grid, wd::kBlock, 0, s.s_main>>>(
-              dk, nullptr, cnt, dst, s.cursor[slot], s.pos[slot], m, t->pseed, t->pmode, B,
-              s.counters);
-        CK(cudaGetLastError());
-        t->launches++;
-      }
+      if (X == 0 && e > 2) TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e - 2));  // owners released e-2
+      if (cnt) TRY(multisplit(s, dk, dv, cnt, slot));
       if (insert) TRY(stage_out(s, io, off, cnt, int(b % kStage), false));  // input slot free
-      wd::FlagPtrs cnt_dst{};
-      for (int d = 0; d < m; ++d) cnt_dst.p[d] = t->peers[d].recv_count[slot] + s.id;
-      wd::publish_kernel<<<1, 32, 0, s.s_main>>>(s.cursor[slot], cnt_dst,
-                                                 flag_ptrs(t, FLAG_READY, s.id), m, e);
-      CK(cudaGetLastError());
-      t->launches++;
+      if (X == 0) {
+        TRY(publish(s, slot, e));
+      } else {                          // this shard's row of T to the host
+        CK(cudaMemcpyAsync(s.hrow[slot], s.cursor[slot], m * 8, cudaMemcpyDeviceToHost, s.s_main));
+        CK(cudaEventRecord(s.ev_row, s.s_main));
+      }
+    }
+    return WD_OK;
+  };
+  // T (staged only): the transposition of P:117 with exact counts — the copy engine pushes
+  // each bucket into its owner's receive region and publishes the counts with the READY
+  // flags; NCCL all-gathers T (rank mode), then one grouped send/recv per peer (an
+  // all-to-all(v)).  The host waits for this batch's row(s) of T first.
+  auto phaseT = [&](uint64_t b) -> wd_status_t {
+    const unsigned long long e = e0 + 1 + b;
+    const int slot = int(e & 1);
+    for (auto& s : t->local) {
+      DeviceGuard g(s.device);
+      CK(cudaEventSynchronize(s.ev_row));
+    }
+    if (X == 1) {
+      for (auto& s : t->local) {
+        DeviceGuard g(s.device);
+        if (e > 2) TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e - 2));   // owners released e-2
+        for (int d = 0; d < m; ++d) {
+          const uint64_t c = std::min<uint64_t>(s.hrow[slot][d], B);
+          if (c)
+            CK(cudaMemcpyAsync(reinterpret_cast<char*>(t->peers[d].recv[slot]) + uint64_t(s.id) * B * isz,
+                               static_cast<char*>(s.send) + uint64_t(d) * B * isz, c * isz,
+                               cudaMemcpyDefault, s.s_main));
+        }
+        TRY(publish(s, slot, e));       // counts + READY after the copies (stream order)
+      }
+      return WD_OK;
+    }
+    // X == 2: the whole T on the host
+    unsigned long long* T = t->local[0].hT[slot];
+    if (all_local) {
+      for (auto& s : t->local)
+        for (int d = 0; d < m; ++d) T[size_t(s.id) * m + d] = s.hrow[slot][d];
+    } else {
+      Shard& s = t->local[0];
+      DeviceGuard g(s.device);
+      NK(g_nccl.AllGather(s.cursor[slot], s.Tdev[slot], m, kNcclUint64, s.comm_fwd, s.s_main));
+      CK(cudaMemcpyAsync(T, s.Tdev[slot], size_t(m) * m * 8, cudaMemcpyDeviceToHost, s.s_main));
+      CK(cudaStreamSynchronize(s.s_main));
+    }
+    for (auto& s : t->local) {          // the receive region must be free: own probe of e-2
+      DeviceGuard g(s.device);
+      if (s.pdone_rec[slot]) CK(cudaStreamWaitEvent(s.s_main, s.ev_pdone[slot], 0));
+    }
+    NK(g_nccl.GroupStart());
+    for (auto& s : t->local) {
+      DeviceGuard g(s.device);
+      for (int d = 0; d < m; ++d) {
+        const uint64_t cs = std::min<uint64_t>(T[size_t(s.id) * m + d], B);   // s -> d
+        const uint64_t cr = std::min<uint64_t>(T[size_t(d) * m + s.id], B);   // d -> s
+        if (cs) NK(g_nccl.Send(static_cast<char*>(s.send) + uint64_t(d) * B * isz, cs * isz,
+                               kNcclUint8, d, s.comm_fwd, s.s_main));
+        if (cr) NK(g_nccl.Recv(reinterpret_cast<char*>(s.self.recv[slot]) + uint64_t(d) * B * isz,
+                               cr * isz, kNcclUint8, d, s.comm_fwd, s.s_main));
+      }
+    }
+    NK(g_nccl.GroupEnd());
+    for (auto& s : t->local) {          // my column of T -> recv_count (InSeg), cursor reset
+      DeviceGuard g(s.device);
+      for (int d = 0; d < m; ++d) s.hcol[slot][d] = T[size_t(d) * m + s.id];
+      CK(cudaMemcpyAsync(s.self.recv_count[slot], s.hcol[slot], m * 8, cudaMemcpyHostToDevice, s.s_main));
+      CK(cudaMemsetAsync(s.cursor[slot], 0, m * 8, s.s_main));
+      CK(cudaEventRecord(s.ev_ready[slot], s.s_main));
     }
     return WD_OK;
   };
@@ -659,26 +902,82 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
     const int slot = int(e & 1);
     for (auto& s : t->local) {
       DeviceGuard g(s.device);
-      TRY(launch_wait(t, s, s.s_probe, FLAG_READY, e));
+      if (X == 2) CK(cudaStreamWaitEvent(s.s_probe, s.ev_ready[slot], 0));
+      else TRY(launch_wait(t, s, s.s_probe, FLAG_READY, e));
       if (insert) {
         const wd::InSeg<true> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
         TRY(launch_probe<true>(t, s, in, wd::OutNone{}, B, s.s_probe));
       } else {
-        // origins consumed the results of the previous query epoch that used this slot
-        if (t->res_used[slot]) TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
         const wd::InSeg<false> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
-        // reverse transposition: results go straight to their origins' result
-        // slots (region s.id of origin d's slot), coalesced remote stores
-        wd::OutPacked out{};
-        out.stride = B;
-        out.shift = __builtin_ctzll(B);
-        for (int d = 0; d < m; ++d) out.seg[d] = t->peers[d].res[slot] + uint64_t(s.id) * B;
-        if (op == OP_ERASE)
-          TRY(launch_probe<false>(t, s, in, wd::OutErase<wd::OutPacked>{out}, B, s.s_probe));
-        else
-          TRY(launch_probe<false>(t, s, in, out, B, s.s_probe));
+        if (X == 0) {
+          // origins consumed the results of the previous query epoch that used this slot
+          if (t->res_used[slot]) TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
+          // reverse transposition: results go straight to their origins' result
+          // slots (region s.id of origin d's slot), coalesced remote stores
+          wd::OutPacked out{};
+          out.stride = B;
+          out.shift = __builtin_ctzll(B);
+          for (int d = 0; d < m; ++d) out.seg[d] = t->peers[d].res[slot] + uint64_t(s.id) * B;
+          if (op == OP_ERASE)
+            TRY(launch_probe<false>(t, s, in, wd::OutErase<wd::OutPacked>{out}, B, s.s_probe));
+          else
+            TRY(launch_probe<false>(t, s, in, out, B, s.s_probe));
+        } else {
+          // staged: results at their receive location in res_stage, then transferred back
+          const wd::OutLocalPacked out{s.res_stage};
+          if (op == OP_ERASE)
+            TRY(launch_probe<false>(t, s, in, wd::OutErase<wd::OutLocalPacked>{out}, B, s.s_probe));
+          else
+            TRY(launch_probe<false>(t, s, in, out, B, s.s_probe));
+        }
       }
-      TRY(launch_signal(t, s, s.s_probe, FLAG_DONE, e));
+      if (X == 2) {
+        CK(cudaEventRecord(s.ev_pdone[slot], s.s_probe));   // recv[slot] may be refilled
+        s.pdone_rec[slot] = true;
+      }
+    }
+    if (!insert && X == 1) {            // reverse transposition with the copy engine
+      for (auto& s : t->local) {
+        DeviceGuard g(s.device);
+        const unsigned long long* col = s.hcol[slot];
+        if (all_local) {
+          for (int d = 0; d < m; ++d) s.hcol[slot][d] = t->local[d].hrow[slot][s.id];
+        } else {                       // my column of T: the counts the senders published
+          CK(cudaMemcpyAsync(s.hcol[slot], s.self.recv_count[slot], m * 8, cudaMemcpyDeviceToHost, s.s_probe));
+          CK(cudaEventRecord(s.ev_col, s.s_probe));
+          CK(cudaEventSynchronize(s.ev_col));
+        }
+        if (t->res_used[slot]) TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
+        for (int d = 0; d < m; ++d) {
+          const uint64_t c = std::min<uint64_t>(col[d], B);
+          if (c)
+            CK(cudaMemcpyAsync(t->peers[d].res[slot] + uint64_t(s.id) * B,
+                               s.res_stage + uint64_t(d) * B, c * 8, cudaMemcpyDefault, s.s_probe));
+        }
+      }
+    }
+    if (!insert && X == 2) {            // reverse transposition with NCCL
+      const unsigned long long* T = t->local[0].hT[slot];
+      for (auto& s : t->local) {        // own result slot free: own unpermute of e-2
+        DeviceGuard g(s.device);
+        if (s.unperm_rec[slot]) CK(cudaStreamWaitEvent(s.s_probe, s.ev_unperm[slot], 0));
+      }
+      NK(g_nccl.GroupStart());
+      for (auto& s : t->local) {
+        DeviceGuard g(s.device);
+        for (int d = 0; d < m; ++d) {
+          const uint64_t cs = std::min<uint64_t>(T[size_t(d) * m + s.id], B);  // answers to d
+          const uint64_t cr = std::min<uint64_t>(T[size_t(s.id) * m + d], B);  // from d
+          if (cs) NK(g_nccl.Send(s.res_stage + uint64_t(d) * B, cs * 8, kNcclUint8, d, s.comm_rev, s.s_probe));
+          if (cr) NK(g_nccl.Recv(s.self.res[slot] + uint64_t(d) * B, cr * 8, kNcclUint8, d, s.comm_rev, s.s_probe));
+        }
+      }
+      NK(g_nccl.GroupEnd());
+    }
+    for (auto& s : t->local) {
+      DeviceGuard g(s.device);
+      if (X == 2) CK(cudaEventRecord(s.ev_done[slot], s.s_probe));
+      else TRY(launch_signal(t, s, s.s_probe, FLAG_DONE, e));
     }
     if (!insert) t->res_used[slot] = e;
     return WD_OK;
@@ -691,7 +990,8 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       const IO& io = ios[r];
       DeviceGuard g(s.device);
       const uint64_t off = std::min(io.n, b * B), cnt = std::min(B, io.n - off);
-      TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e));
+      if (X == 2) CK(cudaStreamWaitEvent(s.s_main, s.ev_done[slot], 0));
+      else TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e));
       if (cnt) {
         wd::DstPtrs src{};
         for (int d = 0; d < m; ++d) src.p[d] = s.self.res[slot] + uint64_t(d) * B;   // local
@@ -703,15 +1003,24 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
         CK(cudaGetLastError());
         t->launches++;
       }
-      TRY(launch_signal(t, s, s.s_main, FLAG_RESC, e));
+      if (X == 2) {
+        CK(cudaEventRecord(s.ev_unperm[slot], s.s_main));
+        s.unperm_rec[slot] = true;
+      } else {
+        TRY(launch_signal(t, s, s.s_main, FLAG_RESC, e));
+      }
       TRY(stage_out(s, io, off, cnt, int(b % kStage), true));
     }
     return WD_OK;
   };
 
   TRY(phaseA(0));
+  if (X) TRY(phaseT(0));
   for (uint64_t b = 0; b < nbt; ++b) {
-    if (b + 1 < nbt) TRY(phaseA(b + 1));
+    if (b + 1 < nbt) {
+      TRY(phaseA(b + 1));
+      if (X) TRY(phaseT(b + 1));
+    }
     TRY(phaseB(b));
     if (!insert) TRY(phaseC(b));
   }
@@ -1007,6 +1316,15 @@ wd_status_t wd_rank_handle(wd_table_t* t, uint8_t out[WD_RANK_HANDLE_BYTES]) {
     memcpy(h.ipc, &ipc, 64);
     h.batch = t->xbatch;
     h.arena_bytes = s.arena_bytes;
+    h.exchange = uint32_t(t->exchange);
+    if (t->exchange == 2 && t->rank == 0) {   // NCCL bootstrap id, only when asked for
+      const NcclApi* a = nccl_api();
+      if (!a) return fail(WD_ERR_NCCL, "%s", g_nccl.why);
+      NcclUid id;
+      NK(a->GetUniqueId(&id));
+      memcpy(h.nccl_id, &id, sizeof id);
+      h.has_nccl_id = 1;
+    }
   }
   memcpy(out, &h, sizeof h);
   return WD_OK;
@@ -1028,6 +1346,12 @@ wd_status_t wd_rank_connect(wd_table_t* t, const uint8_t* handles, wd_allreduce_
       return fail(WD_ERR_INVALID_ARG, "handle %d: bad magic/world/rank order", d);
     if (h.batch != t->xbatch || h.arena_bytes != s.arena_bytes)
       return fail(WD_ERR_INVALID_ARG, "handle %d: batch size differs between ranks", d);
+    if (int(h.exchange) != t->exchange)
+      return fail(WD_ERR_INVALID_ARG, "handle %d: WD_OPT_EXCHANGE differs between ranks", d);
+    if (d == 0 && h.has_nccl_id) {
+      memcpy(t->nccl_id, h.nccl_id, sizeof t->nccl_id);
+      t->have_nccl_id = true;
+    }
     if (d == t->rank) continue;
     cudaIpcMemHandle_t ipc;
     memcpy(&ipc, h.ipc, 64);
@@ -1055,6 +1379,8 @@ void wd_destroy(wd_table_t* t) {
     host_allreduce(t, &one, WD_REDUCE_SUM);
   }
   for (void* p : t->opened) cudaIpcCloseMemHandle(p);
+  if (t->nccl_ready) free_nccl(t);
+  for (auto& s : t->local) free_staged(s);
   for (auto& s : t->local) shard_free(s);
   if (t->loop_stream) cudaStreamDestroy(t->loop_stream);
   delete t;
@@ -1258,6 +1584,15 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       if (v < 0 || v > wd::kMaxShards) return fail(WD_ERR_INVALID_ARG, "slices %lld", (long long)v);
       t->slices = int(v);
       return WD_OK;
+    case WD_OPT_EXCHANGE:
+      if (v < 0 || v > 2) return fail(WD_ERR_INVALID_ARG, "exchange %lld", (long long)v);
+      if (v == 2 && t->mode == MODE_LOOPBACK)
+        return fail(WD_ERR_UNSUPPORTED, "the NCCL exchange needs one GPU per shard; loopback "
+                                        "shards share a device (use 1, the copy engine)");
+      if (t->mode == MODE_RANK && t->connected && int(v) != t->exchange)
+        return fail(WD_ERR_INVALID_ARG, "rank mode: WD_OPT_EXCHANGE is fixed by wd_rank_connect");
+      t->exchange = int(v);
+      return WD_OK;
     default: return fail(WD_ERR_INVALID_ARG, "option %d is read-only or unknown", int(opt));
   }
 }
@@ -1279,6 +1614,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_PART_MODE: return t->pmode;
     case WD_OPT_SPAN: return t->span;
     case WD_OPT_SLICES: return t->slices;
+    case WD_OPT_EXCHANGE: return t->exchange;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;
     case WD_OPT_LOCAL_SHARDS: return int64_t(t->local.size());

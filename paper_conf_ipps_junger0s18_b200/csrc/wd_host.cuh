@@ -108,6 +108,22 @@ struct Shard {
   cudaEvent_t ev_join_probe = nullptr;
   cudaEvent_t ev_fork = nullptr;   // _sharded calls: this shard's caller stream
   bool h2d_pending[kStage] = {};   // the slot's staging buffers have a pending release (ev_free)
+  // staged exchange (WD_OPT_EXCHANGE = 1 copy engine, 2 NCCL): the multisplit writes the
+  // batch into a local send buffer [m][B]; query results are staged in res_stage [m][B]
+  // before the reverse transfer.  hrow / hcol: pinned host copies of this shard's row /
+  // column of T per exchange slot; Tdev: the gathered T (NCCL rank mode)
+  void* send = nullptr;
+  unsigned long long* res_stage = nullptr;
+  uint64_t staged_B = 0;
+  unsigned long long* hrow[2] = {nullptr, nullptr};
+  unsigned long long* hcol[2] = {nullptr, nullptr};
+  unsigned long long* hT[2] = {nullptr, nullptr};
+  unsigned long long* Tdev[2] = {nullptr, nullptr};
+  cudaEvent_t ev_row = nullptr, ev_col = nullptr;
+  cudaEvent_t ev_ready[2] = {}, ev_pdone[2] = {}, ev_done[2] = {}, ev_unperm[2] = {};
+  bool pdone_rec[2] = {}, unperm_rec[2] = {};
+  void* comm_fwd = nullptr;        // ncclComm_t of the forward / reverse transpositions
+  void* comm_rev = nullptr;
   bool l2_held = false;            // holds the device's L2 fetch-granularity setting
 };
 
@@ -150,6 +166,14 @@ struct wd_table {
   void* allreduce_ctx = nullptr;
   bool connected = false;
   cudaStream_t loop_stream = nullptr;       // loopback: one stream for all shards
+  // a8 / a10 transport (WD_OPT_EXCHANGE): 0 fused peer stores in the multisplit / probe
+  // kernels, 1 staged buffers + copy engine (cudaMemcpyAsync of exact counts, the paper's
+  // "asynchronous inter-GPU copies"), 2 staged buffers + NCCL send/recv (all-to-all(v) of
+  // exact counts after an all-gather of T; the north star's NCCL path)
+  int exchange = 0;
+  bool nccl_ready = false;
+  unsigned char nccl_id[128] = {};           // rank mode: rank 0's ncclUniqueId (wd_rank_connect)
+  bool have_nccl_id = false;
 };
 
 namespace wdi {
@@ -312,7 +336,9 @@ wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, 
   X(G, false, wd::InSoA, wd::OutSoA)                          \
   X(G, false, wd::InSoA, wd::OutErase<wd::OutSoA>)            \
   X(G, false, wd::InSeg<false>, wd::OutPacked)                \
-  X(G, false, wd::InSeg<false>, wd::OutErase<wd::OutPacked>)
+  X(G, false, wd::InSeg<false>, wd::OutErase<wd::OutPacked>) \
+  X(G, false, wd::InSeg<false>, wd::OutLocalPacked)          \
+  X(G, false, wd::InSeg<false>, wd::OutErase<wd::OutLocalPacked>)
 #define WD_PROBE_SIG(G, I, IN, OUT) \
   launch_probe_g<G, I, IN, OUT>(wd_table*, Shard&, const IN&, const OUT&, uint64_t, cudaStream_t)
 #define WD_PROBE_EXTERN(G, I, IN, OUT) extern template wd_status_t WD_PROBE_SIG(G, I, IN, OUT);

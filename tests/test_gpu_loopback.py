@@ -144,3 +144,50 @@ def test_loopback_sharded_calls(wd, m):
             assert found == n_local
         with pytest.raises(ValueError):
             t.insert_sharded(keys[:1], vals[:1])
+
+
+@pytest.mark.parametrize("m", [2, 3, 8])
+@pytest.mark.parametrize("exchange", [0, 1])
+def test_loopback_exchange_modes(wd, m, exchange):
+    # WD_OPT_EXCHANGE: fused peer stores (0) and the staged copy-engine transposition (1,
+    # the paper's asynchronous inter-GPU copies) must give identical maps: unique keys over
+    # many batches (epochs wrap both exchange slots), host and device buffers, duplicates,
+    # erase through the reverse path
+    import torch
+    n = 250_007
+    keys, vals = wdgen.unique_keys(n, 81), wdgen.values(n, 82)
+    q = wdgen.interleaved_queries(n, 81)
+    with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=m, exchange=exchange) as t:
+        assert t.get_option(wd.WD_OPT_EXCHANGE) == exchange
+        t.set_option(wd.WD_OPT_BATCH, 20_000)
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0 and t.size() == n
+        hv, hf = gpu_roundtrip(t, keys[:0], vals[:0], q, host=True)
+        er = t.erase(to_dev(q[: n // 2]))
+        torch.cuda.synchronize()
+        assert t.sync() == 0
+    cv, cf = oracle.expected_unique(q, n, 81, 82)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+    assert np.array_equal(hf, cf) and np.array_equal(hv, cv)
+    assert np.array_equal(er.cpu().numpy().astype(bool), cf[: n // 2].astype(bool))
+    dk = wdgen.uniform_keys(300_000, 83) % np.uint32(70_000)
+    dv = wdgen.values(300_000, 84)
+    with wd.Table(capacity_for(70_000, 0.9), group_size=4, loopback_shards=m, exchange=exchange) as t:
+        t.set_option(wd.WD_OPT_BATCH, 30_000)
+        qq = np.arange(71_000, dtype=np.uint32)
+        gv, gf = gpu_roundtrip(t, dk, dv, qq)
+        mo = oracle.Map(300_000, dup_mode=True)
+        mo.insert(dk, dv)
+        assert t.sync() == 0 and t.size() == mo.size()
+    ev, ef = mo.retrieve(qq)
+    assert np.array_equal(gf, ef)
+    assert np.all(mo.pair_status(qq[gf == 1], gv[gf == 1]) >= 1)
+
+
+def test_loopback_rejects_nccl_exchange(wd):
+    with wd.Table(1000, group_size=4, loopback_shards=2) as t:
+        with pytest.raises(wd.WarpDriveError) as ei:
+            t.set_option(wd.WD_OPT_EXCHANGE, 2)
+        assert ei.value.status == wd.WD_ERR_UNSUPPORTED
+        with pytest.raises(wd.WarpDriveError):
+            t.set_option(wd.WD_OPT_EXCHANGE, 3)

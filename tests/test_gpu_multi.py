@@ -25,8 +25,8 @@ needs2 = pytest.mark.skipif(_ndev() < 2, reason="needs >= 2 CUDA devices")
 
 
 @needs2
-@pytest.mark.parametrize("G", [4, 16])
-def test_single_process_multi_gpu_host_input(G):
+@pytest.mark.parametrize("G,exchange", [(4, 0), (16, 0), (16, 1), (16, 2)])
+def test_single_process_multi_gpu_host_input(G, exchange):
     import torch
     import oracle
     import paper_conf_ipps_junger0s18_b200 as wd
@@ -36,7 +36,7 @@ def test_single_process_multi_gpu_host_input(G):
     keys, vals = wdgen.unique_keys(n, KS), wdgen.values(n, VS)
     q = wdgen.interleaved_queries(n, KS)
     torch.cuda.set_device(0)
-    with wd.Table(int(math.ceil(n / 0.9)), m, G) as t:
+    with wd.Table(int(math.ceil(n / 0.9)), m, G, exchange=exchange) as t:
         assert t.get_option(wd.WD_OPT_N_SHARDS) == m
         t.set_option(wd.WD_OPT_BATCH, 1 << 18)           # several batches per shard
         kk = torch.from_numpy(keys.view(np.int32)).pin_memory()
@@ -60,7 +60,8 @@ def test_single_process_multi_gpu_host_input(G):
 
 
 @needs2
-def test_single_process_multi_gpu_sharded_device_input():
+@pytest.mark.parametrize("exchange", [0, 1, 2])
+def test_single_process_multi_gpu_sharded_device_input(exchange):
     import torch
     import paper_conf_ipps_junger0s18_b200 as wd
     import wdgen.gpu as gg
@@ -68,7 +69,7 @@ def test_single_process_multi_gpu_sharded_device_input():
     n_local = 1 << 22
     n = n_local * m
     torch.cuda.set_device(0)
-    with wd.Table(int(math.ceil(n / 0.95)), m, 16) as t:
+    with wd.Table(int(math.ceil(n / 0.95)), m, 16, exchange=exchange) as t:
         keys, vals, q, vo, fo, st = [], [], [], [], [], []
         for r in range(m):
             with torch.cuda.device(r):
@@ -99,7 +100,7 @@ def _free_port():
     return p
 
 
-def _rank_worker(rank, world, port, q, n_local, G):
+def _rank_worker(rank, world, port, q, n_local, G, exchange):
     try:
         import torch
         import torch.distributed as dist
@@ -113,7 +114,7 @@ def _rank_worker(rank, world, port, q, n_local, G):
         keys = gg.unique_keys(n_local, KS, start=rank * n_local)
         vals = gg.values(n_local, VS, start=rank * n_local)
         t = wd.Table(int(math.ceil(n / 0.95)), group_size=G, rank=rank, world=world,
-                     batch=1 << 20)
+                     batch=1 << 20, exchange=exchange)
         t.insert(keys, vals)
         qk = gg.interleaved_queries(n, KS, start=2 * rank * n_local, count=2 * n_local)
         vo = torch.empty(2 * n_local, dtype=torch.int32, device="cuda")
@@ -132,14 +133,14 @@ def _rank_worker(rank, world, port, q, n_local, G):
 
 
 @needs2
-@pytest.mark.parametrize("G", [4, 16])
-def test_rank_mode_physical_gpus(G):
+@pytest.mark.parametrize("G,exchange", [(4, 0), (16, 0), (16, 1), (16, 2)])
+def test_rank_mode_physical_gpus(G, exchange):
     import torch.multiprocessing as mp
     world = min(_ndev(), 8)
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_rank_worker, args=(r, world, port, q, 3_000_017, G))
+    procs = [ctx.Process(target=_rank_worker, args=(r, world, port, q, 3_000_017, G, exchange))
              for r in range(world)]
     for p in procs:
         p.start()

@@ -21,7 +21,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, q, n_local, batch, G):
+def _worker(rank, world, port, q, n_local, batch, G, exchange=0):
     try:
         import torch
         import torch.distributed as dist
@@ -36,7 +36,7 @@ def _worker(rank, world, port, q, n_local, batch, G):
         keys = wdgen.unique_keys(n_local, seed, start=rank * n_local)
         vals = wdgen.values(n_local, seed + 1, start=rank * n_local)
         cap = int(np.ceil(world * n_local / 0.9))
-        t = wd.Table(cap, group_size=G, rank=rank, world=world, batch=batch)
+        t = wd.Table(cap, group_size=G, rank=rank, world=world, batch=batch, exchange=exchange)
         dk = torch.from_numpy(keys.view(np.int32)).cuda()
         dv = torch.from_numpy(vals.view(np.int32)).cuda()
         t.insert(dk, dv)
@@ -62,15 +62,16 @@ def _worker(rank, world, port, q, n_local, batch, G):
         q.put((rank, traceback.format_exc()))
 
 
-@pytest.mark.parametrize("G", [4])
-def test_rank_mode_two_processes_one_gpu(G):
+@pytest.mark.parametrize("G,exchange", [(4, 0), (4, 1), (16, 1)])
+def test_rank_mode_two_processes_one_gpu(G, exchange):
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, 50_000, 8_192, G)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, 50_000, 8_192, G, exchange))
+             for r in range(2)]
     for p in procs:
         p.start()
     res = dict(q.get(timeout=300) for _ in procs)
