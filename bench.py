@@ -51,11 +51,13 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n-log2", type=int, default=28, help="pairs per GPU (config 2: 28)")
+    ap.add_argument("--n-log2", type=int, default=None,
+                    help="config 2: pairs per GPU (28); config 3: 2^n - [n = 32] pairs in total (32); "
+                         "config 4: table keys (31); config 5: draws per GPU (30)")
     ap.add_argument("--alpha", type=float, default=0.95)
-    ap.add_argument("--group-size", type=int, default=16,
-                    help="|g| (config 2 sweeps 1-32; 16 is the fastest at alpha 0.95 on B200, "
-                         "profiles/r01_sweep.jsonl)")
+    ap.add_argument("--group-size", type=int, default=None,
+                    help="|g| (config 2: 16, the fastest at alpha 0.95 on B200, "
+                         "profiles/r01_sweep.jsonl; config 3: 4; config 4: 16; config 5: 8)")
     ap.add_argument("--kif", type=int, default=0, help="keys in flight per group (0=default)")
     ap.add_argument("--probe-mode", type=int, default=None,
                     help="0: auto; 1: cooperative group per window (Fig. 3); 2: lane-window")
@@ -70,7 +72,21 @@ def parse():
                          "the ranks (default: weak, 2^n-log2 pairs per GPU)")
     ap.add_argument("--sweep", action="store_true",
                     help="extra lines: config-2 alpha x |g| sweep (not the headline)")
-    return ap.parse_args()
+    ap.add_argument("--config", type=int, default=2, choices=[2, 3, 4, 5],
+                    help="BASELINE config: 2 (default headline; weak, n pairs per GPU), "
+                         "3 (2^32 - 1 unique pairs in total, strong), 4 (query mix on a 2^31-key "
+                         "table, 2^32 queries at 0/50/100%% hits), 5 (uniform draws with "
+                         "duplicates streamed from pinned host memory, per GPU)")
+    ap.add_argument("--exchange", type=int, default=0, choices=[0, 1, 2],
+                    help="N > 1 transposition: 0 fused peer stores, 1 copy engine, 2 NCCL")
+    ap.add_argument("--batch-log2", type=int, default=None,
+                    help="items per shard per cascade batch (default 24, P:197)")
+    args = ap.parse_args()
+    if args.n_log2 is None:
+        args.n_log2 = {2: 28, 3: 32, 4: 31, 5: 30}[args.config]
+    if args.group_size is None:
+        args.group_size = {2: 16, 3: 4, 4: 16, 5: 8}[args.config]
+    return args
 
 
 # ----------------------------------------------------------------------------- clocks
@@ -220,44 +236,321 @@ def workload_config(args, world):
             "global_batch": n * world, "pairs_per_gpu": n, "alpha": args.alpha,
             "group_size": args.group_size,
             "parallelism": f"keyspace-shard{world}" if world > 1 else "single",
+            "exchange": ["fused peer stores", "copy engine", "NCCL"][args.exchange] if world > 1 else None,
             "l2": "inputs (2 x 2^%d x 4 B) and table exceed the 126 MB L2; no flush" % args.n_log2}
+
+
+def make_config(args, world):
+    """the `config` object of the JSON line — identical for our arm and the reference arm"""
+    if args.config == 2:
+        return workload_config(args, world)
+    G, alpha = args.group_size, args.alpha
+    if args.config == 3:
+        n_total = (1 << args.n_log2) - (1 if args.n_log2 == 32 else 0)
+        size = "2^32 - 1, C14" if args.n_log2 == 32 else f"2^{args.n_log2}"
+        wl = (f"config3: {n_total} unique u32 pairs in total ({size}) hash-partitioned over "
+              f"the GPUs, load {alpha}, |g|={G}; step = fill + insert all + retrieve all")
+    elif args.config == 4:
+        wl = (f"config4: table of 2^{args.n_log2} unique keys (load {alpha}, |g|={G}); "
+              f"2^{args.n_log2 + 1} queries at 0 / 50 / 100 % hits each (reverse exchange + "
+              f"unpermute); step = the three query batches")
+    else:
+        N = (1 << args.n_log2) * world
+        expect = 2**32 * (1 - math.exp(-N / 2**32))
+        wl = (f"config5: 2^{args.n_log2} uniform draws WITH replacement per GPU ({N} in total) "
+              f"in pinned host memory, streamed (a11) into a table sized for the expected "
+              f"{expect:.0f} distinct keys at load {alpha}, |g|={G}; step = fill + insert all + "
+              f"retrieve all back to pinned host memory")
+    return {"workload": wl, "baseline_config": args.config, "group_size": G, "alpha": alpha,
+            "parallelism": f"keyspace-shard{world}" if world > 1 else "single",
+            "exchange": ["fused peer stores", "copy engine", "NCCL"][args.exchange] if world > 1 else None,
+            "l2": "inputs and table exceed the 126 MB L2; no flush"}
 
 
 # ----------------------------------------------------------------------------- reference arm
 def run_reference(args):
-    """--impl reference: the oracle (this tier's reference arm) on the host cores, on the
-    same config/metric; each step a bounded sample (2^22 inserts + 2^22 queries)."""
+    """--impl reference: the oracle (this tier's reference arm: the single-threaded C
+    dictionary of oracle/) on one host core, timed as it stands on a BOUNDED sample of the
+    same config's workload per step (same generator, same metric, same `config` object):
+    configs 2 / 3: 2^22 unique inserts + 2^22 hit queries; config 4: 3 x 2^23 queries (0 / 50
+    / 100 % hits) on a 2^22-key table; config 5: 2^22 uniform draws with duplicates, inserted
+    and queried back.  Under torchrun only rank 0 runs."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    import numpy as np
     import oracle
     import wdgen
     n = 1 << 22
-    keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
     times = []
+    if args.config in (2, 3):
+        keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
+        sample = f"2^22 unique inserts + 2^22 hit queries per step (config-{args.config} keys, generator indices [0, 2^22))"
+        ops = 2 * n
+    elif args.config == 4:
+        keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
+        qs = [wdgen.mixed_queries(n, 2 * n, h, KEY_SEED)[0] for h in (0.0, 0.5, 1.0)]
+        sample = "2^22-key table (untimed insert) + 3 x 2^23 queries at 0 / 50 / 100 % hits per step"
+        ops = 6 * n
+    else:
+        keys, vals = wdgen.uniform_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
+        sample = "2^22 uniform draws with replacement (duplicate mode) inserted + queried back per step"
+        ops = 2 * n
     for it in range(args.warmup + args.steps):
-        m = oracle.Map(n)
-        t0 = time.perf_counter()
-        m.insert(keys, vals)
-        v, f = m.retrieve(keys)
+        m = oracle.Map(n, dup_mode=args.config == 5)
+        if args.config == 4:
+            m.insert(keys, vals)
+            t0 = time.perf_counter()
+            for q in qs:
+                m.retrieve(q)
+        else:
+            t0 = time.perf_counter()
+            m.insert(keys, vals)
+            m.retrieve(keys)
         dt = time.perf_counter() - t0
         m.close()
         if it >= args.warmup:
             times.append(dt)
     t = sum(times) / len(times)
-    val = 2 * n / t / 1e9
+    val = ops / t / 1e9
+    scaling = "weak" if args.config in (2, 5) and not args.strong else "strong"
     line = {"metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
-            "higher_is_better": True, "scaling": "strong" if args.strong else "weak",
+            "higher_is_better": True, "scaling": scaling,
             "vs_baseline": None, "dtype": "u32", "data": "synthetic", "impl": "reference",
-            "config": dict(workload_config(args, args.gpus),
-                           reference_sample="bounded 2^22 unique inserts + 2^22 hit queries "
-                                            "per step, single-threaded C oracle"),
+            "config": make_config(args, args.gpus),
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": "2^22 unique inserts + 2^22 hit queries per step"},
+                             "sample": sample + ", single-threaded C oracle (oracle/wd_oracle.c)"},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- configs 3-5
+def _setup_dist(args):
+    import torch
+    import torch.distributed as dist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    assert world == args.gpus or world == 1, "launch N>1 with torchrun --nproc-per-node N"
+    dev = 0 if args.same_device else local_rank
+    torch.cuda.set_device(dev)
+    if world > 1:
+        backend = "gloo" if args.same_device else args.dist_backend
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group(backend)
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+    return torch, dist, world, rank, dev, barrier
+
+
+def _make_table(wd, args, capacity_total, world, rank):
+    kw = {}
+    if args.batch_log2 is not None:
+        kw["batch"] = 1 << args.batch_log2
+    if world > 1:
+        t = wd.Table(capacity_total, group_size=args.group_size, rank=rank, world=world,
+                     exchange=args.exchange, **kw)
+    else:
+        t = wd.Table(capacity_total, 1, args.group_size, **kw)
+    if args.kif:
+        t.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, args.kif)
+    return t
+
+
+def _phases(table, wd, fn, steps=1):
+    """one instrumented repetition of fn (not the timed region): per-phase CUDA-event ms"""
+    table.phase_times()
+    table.set_option(wd.WD_OPT_PHASE_TIMING, 1)
+    for _ in range(steps):
+        fn()
+    out = table.phase_times()
+    table.set_option(wd.WD_OPT_PHASE_TIMING, 0)
+    return {k: round(v[0] / steps, 4) for k, v in out.items() if v[1]}
+
+
+def _nvlink(world, bytes_per_op, ops_per_rank, phase_ms):
+    """NVLink bytes of a cascade call per rank and their rate over the phase that moves them
+    (fused exchange: inside the multisplit / probe; staged: the exchange / reverse phase),
+    against NVLink 5's 900 GB/s per direction per GPU"""
+    if world == 1 or not phase_ms:
+        return None
+    b = bytes_per_op * (world - 1) / world * ops_per_rank
+    gbs = b / (phase_ms * 1e-3) / 1e9
+    return {"bytes_per_op": bytes_per_op * (world - 1) / world, "bytes_per_rank": b,
+            "phase_ms": phase_ms, "GBps_per_gpu": gbs, "frac_of_900GBps": gbs / 900.0}
+
+
+def run_config(args):
+    """BASELINE configs 3, 4, 5 at N GPUs (torchrun, one process per GPU; rank mode).
+    Inputs are device-resident (3, 4) or pinned host memory (5), generated by the seeded
+    generator; every query of the measured configuration is checked against the closed form
+    (3, 4) or the drawn pairs (5, N = 1) after the warm-up."""
+    import numpy as np  # noqa: F401
+    torch, dist, world, rank, dev, barrier = _setup_dist(args)
+    import paper_conf_ipps_junger0s18_b200 as wd
+    import wdgen.gpu as gg
+    from paper_conf_ipps_junger0s18_b200.dist import max_over_ranks
+    ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+    stream = torch.cuda.current_stream()
+    G, alpha = args.group_size, args.alpha
+    info, checks = {}, {}
+    if args.config == 3:
+        # 2^32 pairs -> n = 2^32 - 1 unique keys (C14), contiguous 1/N index slices
+        n_total = (1 << args.n_log2) - (1 if args.n_log2 == 32 else 0)
+        lo, hi = n_total * rank // world, n_total * (rank + 1) // world
+        n = hi - lo
+        table = _make_table(wd, args, int(math.ceil(n_total / alpha)), world, rank)
+        keys, vals = gg.unique_keys(n, KEY_SEED, start=lo), gg.values(n, VAL_SEED, start=lo)
+        vout = torch.empty(n, dtype=torch.int32, device="cuda")
+        fout = torch.empty(n, dtype=torch.uint8, device="cuda")
+
+        def step(m=None):
+            table.clear(stream)
+            if m: m[0].record(stream)
+            table.insert(keys, vals, stream)
+            if m: m[1].record(stream)
+            table.retrieve(keys, vout, fout, stream)
+            if m: m[2].record(stream)
+        ops_total = 2 * n_total
+        scaling = "strong"
+    elif args.config == 4:
+        n_table = 1 << args.n_log2
+        lo, hi = n_table * rank // world, n_table * (rank + 1) // world
+        q_total = 2 * n_table
+        nq = q_total // world
+        table = _make_table(wd, args, int(math.ceil(n_table / alpha)), world, rank)
+        k0, v0 = gg.unique_keys(hi - lo, KEY_SEED, start=lo), gg.values(hi - lo, VAL_SEED, start=lo)
+        table.insert(k0, v0, stream)
+        torch.cuda.synchronize()
+        del k0, v0
+        qs = {}
+        for h in (0.0, 0.5, 1.0):
+            q = torch.empty(nq, dtype=torch.int32, device="cuda")
+            hits = torch.empty(nq, dtype=torch.uint8, device="cuda")
+            gg.mixed_queries(n_table, nq, h, KEY_SEED, start=rank * nq, out=q, hits=hits)
+            qs[h] = (q, hits)
+        vout = torch.empty(nq, dtype=torch.int32, device="cuda")
+        fout = torch.empty(nq, dtype=torch.uint8, device="cuda")
+
+        def step(m=None):
+            for i, h in enumerate((0.0, 0.5, 1.0)):
+                if m: m[i].record(stream)
+                table.retrieve(qs[h][0], vout, fout, stream)
+            if m: m[3].record(stream)
+        ops_total = 3 * q_total
+        scaling = "strong"
+    else:
+        per = 1 << args.n_log2
+        N = per * world
+        expect = 2**32 * (1 - math.exp(-N / 2**32))
+        table = _make_table(wd, args, int(math.ceil(expect / alpha)), world, rank)
+        if args.batch_log2 is None and world == 1:
+            table.set_option(wd.WD_OPT_BATCH, 1 << 22)
+        dk = gg.uniform_keys(per, KEY_SEED, start=rank * per)
+        dv = gg.values(per, VAL_SEED, start=rank * per)
+        hk = torch.empty(per, dtype=torch.int32, pin_memory=True)
+        hv = torch.empty(per, dtype=torch.int32, pin_memory=True)
+        hk.copy_(dk)
+        hv.copy_(dv)
+        hvo = torch.empty(per, dtype=torch.int32, pin_memory=True)
+        hfo = torch.empty(per, dtype=torch.uint8, pin_memory=True)
+
+        def step(m=None):
+            table.clear(stream)
+            if m: m[0].record(stream)
+            table.insert(hk, hv, stream)
+            if m: m[1].record(stream)
+            table.retrieve(hk, hvo, hfo, stream)
+            if m: m[2].record(stream)
+        ops_total = 2 * N
+        scaling = "weak"
+
+    # ---- warm-up + every-query check of the measured configuration
+    nmarks = 4 if args.config == 4 else 3
+    for _ in range(max(1, args.warmup)):
+        step()
+    barrier()
+    st = table.sync()
+    assert st == 0, f"device-side status {st}: {wd._lib.wd_last_error_message()}"
+    if args.config == 3:
+        assert table.size() == n_total
+        bad, first, found = gg.check_unique(keys, vout, fout, n_total, KEY_SEED, VAL_SEED)
+        assert bad == 0 and found == n, (bad, first, found)
+        checks = {"queries_checked": n, "mismatches": bad, "kind": "closed form, every query"}
+    elif args.config == 4:
+        found = {}
+        for h in (0.0, 0.5, 1.0):
+            table.retrieve(qs[h][0], vout, fout, stream)
+            bad, first, f = gg.check_unique(qs[h][0], vout, fout, n_table, KEY_SEED, VAL_SEED)
+            assert bad == 0 and bool((fout == qs[h][1]).all()), (h, bad, first)
+            found[str(h)] = f
+        checks = {"queries_checked": 3 * nq, "mismatches": 0, "found": found,
+                  "kind": "closed form + generator hit flag, every query"}
+    else:
+        size = table.size()
+        assert abs(size - expect) < 6 * math.sqrt(expect) + 16, (size, expect)
+        assert bool((hfo == 1).all())
+        checks = {"size": size, "expected_distinct": expect, "all_found": True}
+        if world == 1:
+            uniq = torch.unique(dk.to(torch.int64) & 0xFFFFFFFF)
+            assert size == uniq.numel()
+            pairs = torch.sort(((dk.to(torch.int64) & 0xFFFFFFFF) << 32) | (dv.to(torch.int64) & 0xFFFFFFFF)).values
+            got = ((dk.to(torch.int64) & 0xFFFFFFFF) << 32) | (hvo.cuda().to(torch.int64) & 0xFFFFFFFF)
+            pp = torch.searchsorted(pairs, got).clamp(max=pairs.numel() - 1)
+            assert bool((pairs[pp] == got).all())
+            checks.update(distinct_exact=True, values_checked=per, kind="every returned value among the drawn pairs")
+            del uniq, pairs, got, pp
+        del dk, dv
+
+    # ---- timed region
+    launches0 = table.launches
+    marks = [[ev() for _ in range(nmarks)] for _ in range(args.steps)]
+    e0, e1 = ev(), ev()
+    with ClockSampler(dev) as clk:
+        barrier()
+        e0.record(stream)
+        for k in range(args.steps):
+            step(marks[k])
+        e1.record(stream)
+        barrier()
+    launches = table.launches - launches0
+    t_ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+    sub = [max_over_ranks(sum(mk[i].elapsed_time(mk[i + 1]) for mk in marks) / args.steps)
+           for i in range(nmarks - 1)]
+    assert table.sync() == 0
+    value = ops_total / (t_ms * 1e-3) / 1e9
+    phases = _phases(table, wd, lambda: step())
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": t_ms, "higher_is_better": True,
+            "scaling": scaling, "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic (seeded generator)", "config": make_config(args, world),
+            "clocks": clk.summary(), "gpu_launches": launches, "checks": checks,
+            "phases_ms_rank0": phases}
+    if args.config in (3, 5):
+        nn = n_total if args.config == 3 else N
+        line["insert_gops"] = nn / (sub[0] * 1e-3) / 1e9
+        line["query_gops"] = nn / (sub[1] * 1e-3) / 1e9
+        line["nvlink"] = {"insert": _nvlink(world, 8, nn / world, phases.get("multisplit") if args.exchange == 0 else phases.get("exchange")),
+                          "query": _nvlink(world, 12, nn / world, phases.get("probe") if args.exchange == 0 else phases.get("reverse"))}
+    else:
+        line["mix"] = {str(h): {"query_gops": q_total / (sub[i] * 1e-3) / 1e9, "ms": sub[i]}
+                       for i, h in enumerate((0.0, 0.5, 1.0))}
+        line["query_gops"] = value
+    if args.config == 5:
+        line["e2e"] = {"value": value, "unit": UNIT, "h2d_bytes_per_step": 12 * per,
+                       "d2h_bytes_per_step": 5 * per,
+                       "note": "config 5 IS the host-streamed path: value is end to end"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    table.close()
+    if world > 1:
+        dist.destroy_process_group()
 
 
 # ----------------------------------------------------------------------------- our arm
@@ -265,6 +558,8 @@ def main():
     args = parse()
     if args.impl == "reference":
         return run_reference(args)
+    if args.config != 2:
+        return run_config(args)
     import numpy as np
     import torch
     import torch.distributed as dist
@@ -290,12 +585,7 @@ def main():
     n = (1 << args.n_log2) // (world if args.strong else 1)
     G = args.group_size
     cap_local = int(math.ceil(n / args.alpha))
-    if world > 1:
-        table = wd.Table(cap_local * world, group_size=G, rank=rank, world=world)
-    else:
-        table = wd.Table(cap_local, 1, G)
-    if args.kif:
-        table.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, args.kif)
+    table = _make_table(wd, args, cap_local * world, world, rank)
     if args.probe_mode is not None:
         table.set_option(wd.WD_OPT_PROBE_MODE, args.probe_mode)
 
@@ -369,6 +659,12 @@ def main():
     ops = 2 * n * world
     value = ops / (t_ms * 1e-3) / 1e9
     assert table.sync() == 0
+    # per-phase decomposition (Fig. 11) of one more, instrumented step (not the timed ones)
+    phases = _phases(table, wd, lambda: step())
+    nvlink = None
+    if world > 1:
+        nvlink = {"insert": _nvlink(world, 8, n, phases.get("multisplit") if args.exchange == 0 else phases.get("exchange")),
+                  "query": _nvlink(world, 12, n, phases.get("probe") if args.exchange == 0 else phases.get("reverse"))}
 
     # ---- roofline of the dominant kernel (single GPU: one launch per call)
     pc = probe_cost(args.alpha, G)
@@ -496,12 +792,13 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_ms,
             "higher_is_better": True, "scaling": "strong" if args.strong else "weak",
             "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-            "config": dict(workload_config(args, world),
-                           capacity_per_gpu=table.shard_capacity(0)),
+            "config": make_config(args, world),
+            "capacity_per_gpu": table.shard_capacity(0),
             "insert_gops": n * world / (ins_ms * 1e-3) / 1e9,
             "query_gops": n * world / (qry_ms * 1e-3) / 1e9,
             "fill_ms": fill_ms,
             "roofline": roofline, "cpu_baseline": cpu,
+            "phases_ms_rank0": phases, "nvlink": nvlink,
             "clocks": clk.summary(), "e2e": e2e, "gpu_launches": launches,
             "gpu_launches_per_step": launches / args.steps,
         }

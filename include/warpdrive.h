@@ -243,6 +243,8 @@ typedef enum {
                                   rank mode: set before wd_rank_handle).  NCCL is loaded at
                                   run time (libnccl.so.2).
                                 Results are identical in all three modes. */
+    WD_OPT_PHASE_TIMING = 13, /* 1: record CUDA events around every phase of every call (see
+                                wd_phase_times); 0 (default): off */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */
@@ -257,6 +259,23 @@ typedef enum {
 
 wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t value);
 int64_t     wd_get_option(wd_table_t* t, wd_option_t opt);   /* INT64_MIN on error */
+
+/* ------------------------------------------------------------------ phase timing --- */
+/* The per-phase decomposition of Fig. 11.  With WD_OPT_PHASE_TIMING = 1 every
+ * phase of every batch is bracketed by CUDA events on the stream it runs on; this call
+ * synchronizes, writes the summed milliseconds (and the number of intervals) per phase
+ * since the last call, and resets.  Phases on different streams overlap, so the sum is
+ * not the wall time.  Indices: */
+#define WD_PHASE_H2D 0         /* a11: host -> device copies of the input */
+#define WD_PHASE_GROUP 1       /* slice grouping of a bulk insert (histogram, scan, multisplit) */
+#define WD_PHASE_MULTISPLIT 2  /* a6 (fused mode: includes the transposition a8) */
+#define WD_PHASE_EXCHANGE 3    /* a8 staged: copy engine / NCCL send+recv */
+#define WD_PHASE_PROBE 4       /* a3 / a4 / a9 probe kernels (fused mode: includes a10's push) */
+#define WD_PHASE_REVERSE 5     /* a10 staged: results back to their origins */
+#define WD_PHASE_UNPERMUTE 6   /* a10: gather into input order */
+#define WD_PHASE_D2H 7         /* a11: device -> host copies of the results */
+#define WD_N_PHASES 8
+wd_status_t wd_phase_times(wd_table_t* t, double ms_out[WD_N_PHASES], uint64_t count_out[WD_N_PHASES]);
 
 /* ------------------------------------------------------------------ diagnostics ---- */
 wd_status_t wd_last_error(void);

@@ -32,6 +32,8 @@ WD_OPT_GROUP_SIZE, WD_OPT_P_MAX, WD_OPT_BATCH, WD_OPT_SERIAL = 0, 1, 2, 3
 WD_OPT_KEYS_IN_FLIGHT, WD_OPT_PART_SEED, WD_OPT_PART_MODE, WD_OPT_PROBE_MODE = 4, 5, 6, 7
 WD_OPT_KERNEL_FLAGS, WD_OPT_SLOTS_PER_LANE, WD_OPT_SPAN, WD_OPT_SLICES = 8, 9, 10, 11
 WD_OPT_EXCHANGE = 12
+WD_OPT_PHASE_TIMING = 13
+PHASES = ["h2d", "group", "multisplit", "exchange", "probe", "reverse", "unpermute", "d2h"]
 EXCHANGE_FUSED, EXCHANGE_COPY, EXCHANGE_NCCL = 0, 1, 2
 WD_OPT_N_SHARDS, WD_OPT_RANK, WD_OPT_LOCAL_SHARDS, WD_OPT_LAUNCHES = 100, 101, 102, 103
 WD_OPT_GROUP_SIZE_USED = 104
@@ -45,7 +47,7 @@ EXPORTS = ["wd_create", "wd_create_loopback", "wd_create_rank", "wd_rank_handle"
            "wd_destroy", "wd_clear", "wd_insert", "wd_retrieve", "wd_size", "wd_capacity",
            "wd_sync", "wd_set_option", "wd_get_option", "wd_last_error", "wd_error_string",
            "wd_last_error_message", "wd_shard_capacity", "wd_dump", "wd_counters", "wd_erase",
-           "wd_rebuild", "wd_insert_sharded", "wd_retrieve_sharded"]
+           "wd_rebuild", "wd_insert_sharded", "wd_retrieve_sharded", "wd_phase_times"]
 
 
 class WarpDriveError(RuntimeError):
@@ -92,6 +94,7 @@ def _load():
         "wd_rebuild": ([p, C.c_uint32, p], i32),
         "wd_insert_sharded": ([p, p, p, p, p], i32),
         "wd_retrieve_sharded": ([p, p, p, p, p, p], i32),
+        "wd_phase_times": ([p, p, p], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -325,6 +328,14 @@ class Table:
         return {"new": int(out[0]), "failed": int(out[1]), "reserved": int(out[2]),
                 "exchange_errors": int(out[3]), "last_failed_key": int(out[4]),
                 "erased": int(out[5])}
+
+    def phase_times(self) -> dict:
+        """Per-phase CUDA-event milliseconds since the last call (WD_OPT_PHASE_TIMING = 1);
+        synchronizes and resets.  {phase: (ms, intervals)}"""
+        ms = (C.c_double * len(PHASES))()
+        cnt = (C.c_uint64 * len(PHASES))()
+        _check(_lib.wd_phase_times(self._h, C.addressof(ms), C.addressof(cnt)))
+        return {p: (ms[i], int(cnt[i])) for i, p in enumerate(PHASES)}
 
     @property
     def launches(self) -> int:

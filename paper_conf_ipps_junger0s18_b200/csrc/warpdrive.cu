@@ -18,6 +18,7 @@
 #include "wd_host.cuh"
 
 #include <dlfcn.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <mutex>
 
@@ -97,6 +98,42 @@ const NcclApi* nccl_api() {
       return fail(WD_ERR_NCCL, "%s: %s (%s:%d)", #x, g_nccl.GetErrorString(r_), __FILE__, \
                   __LINE__);                                                               \
   } while (0)
+
+// ------------------------------------------------------------------ phases: events + NVTX
+// WD_OPT_PHASE_TIMING = 1 records a CUDA-event pair around every phase of every batch, on
+// the stream the phase runs on (the decomposition of Fig. 11); wd_phase_times
+// sums them.  NVTX ranges mark the host-side issue of every call and phase (for nsys /
+// ncu --nvtx; no-ops without a tool attached).
+struct Nvtx {
+  explicit Nvtx(const char* name) { nvtxRangePushA(name); }
+  ~Nvtx() { nvtxRangePop(); }
+};
+struct Ph { cudaEvent_t a = nullptr; int phase = 0, device = 0; cudaStream_t st = nullptr; };
+cudaEvent_t ph_event(wd_table* t, int device) {
+  auto& pool = t->ph_pool[device];
+  if (!pool.empty()) {
+    cudaEvent_t e = pool.back();
+    pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  if (cudaEventCreate(&e) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+  return e;
+}
+Ph ph_begin(wd_table* t, int phase, int device, cudaStream_t st) {
+  Ph p;
+  if (!t->phase_on) return p;
+  p.a = ph_event(t, device);
+  if (p.a && cudaEventRecord(p.a, st) != cudaSuccess) { cudaGetLastError(); p.a = nullptr; }
+  p.phase = phase; p.device = device; p.st = st;
+  return p;
+}
+void ph_end(wd_table* t, const Ph& p) {
+  if (!p.a) return;
+  cudaEvent_t b = ph_event(t, p.device);
+  if (!b || cudaEventRecord(b, p.st) != cudaSuccess) { cudaGetLastError(); return; }
+  t->ph_recs.push_back({p.phase, p.device, p.a, b});
+}
 
 // ------------------------------------------------------------------ L2 fetch granularity
 // Random 32-byte windows: do not let L2 promote a sector miss to a 64/128-byte DRAM fetch
@@ -421,8 +458,8 @@ struct IO {
 };
 
 // stage batch b's input of `io` into device memory; returns device pointers
-wd_status_t stage_in(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slot, bool with_vals,
-                     const uint32_t** dk, const uint32_t** dv) {
+wd_status_t stage_in(wd_table* t, Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slot,
+                     bool with_vals, const uint32_t** dk, const uint32_t** dv) {
   DeviceGuard g(s.device);
   // the slot's staging buffers (input and output) may still be used by an earlier batch —
   // of this call or of an earlier call on any stream: both the copy-in and the kernel that
@@ -448,8 +485,10 @@ wd_status_t stage_in(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slo
     hv = hv ? s.pin_vals[slot] : nullptr;
   }
   if (cnt) {
+    const Ph ph = ph_begin(t, wd::PH_H2D, s.device, s.s_h2d);
     CK(cudaMemcpyAsync(s.st_keys[slot], hk, cnt * 4, cudaMemcpyHostToDevice, s.s_h2d));
     if (hv) CK(cudaMemcpyAsync(s.st_vals[slot], hv, cnt * 4, cudaMemcpyHostToDevice, s.s_h2d));
+    ph_end(t, ph);
   }
   CK(cudaEventRecord(s.ev_h2d[slot], s.s_h2d));
   CK(cudaStreamWaitEvent(s.s_main, s.ev_h2d[slot], 0));
@@ -471,7 +510,7 @@ void out_ptrs(Shard& s, const IO& io, uint64_t off, int slot, uint32_t** dv, uin
 
 // after the kernel that consumed slot `slot` (recorded on s_main): release staging;
 // for host outputs copy results back (pageable: through the pinned bounce, synchronously)
-wd_status_t stage_out(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slot, bool query) {
+wd_status_t stage_out(wd_table* t, Shard& s, const IO& io, uint64_t off, uint64_t cnt, int slot, bool query) {
   DeviceGuard g(s.device);
   CK(cudaEventRecord(s.ev_kdone[slot], s.s_main));
   if (!query || io.kout == PK_DEVICE) {
@@ -482,14 +521,17 @@ wd_status_t stage_out(Shard& s, const IO& io, uint64_t off, uint64_t cnt, int sl
     return WD_OK;
   }
   CK(cudaStreamWaitEvent(s.s_d2h, s.ev_kdone[slot], 0));
+  const Ph ph = ph_begin(t, wd::PH_D2H, s.device, s.s_d2h);
   if (io.kout == PK_PINNED) {
     if (io.vout && cnt) CK(cudaMemcpyAsync(io.vout + off, s.st_vout[slot], cnt * 4, cudaMemcpyDeviceToHost, s.s_d2h));
     if (io.fout && cnt) CK(cudaMemcpyAsync(io.fout + off, s.st_fout[slot], cnt, cudaMemcpyDeviceToHost, s.s_d2h));
+    ph_end(t, ph);
     CK(cudaEventRecord(s.ev_free[slot], s.s_d2h));
     s.h2d_pending[slot] = true;
   } else {
     if (io.vout && cnt) CK(cudaMemcpyAsync(s.pin_vout[slot], s.st_vout[slot], cnt * 4, cudaMemcpyDeviceToHost, s.s_d2h));
     if (io.fout && cnt) CK(cudaMemcpyAsync(s.pin_fout[slot], s.st_fout[slot], cnt, cudaMemcpyDeviceToHost, s.s_d2h));
+    ph_end(t, ph);
     CK(cudaEventRecord(s.ev_free[slot], s.s_d2h));
     s.h2d_pending[slot] = true;
     CK(cudaEventSynchronize(s.ev_free[slot]));
@@ -572,6 +614,7 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
   const int ms_grid_cap = t->sm_count * blocks_per_sm(wd::multisplit_kernel<true>);
   for (uint64_t off = 0; off < io.n; off += kChunkPairs) {
     const uint64_t cnt = std::min(kChunkPairs, io.n - off);
+    const Ph pg = ph_begin(t, wd::PH_GROUP, s.device, st);
     CK(cudaMemsetAsync(counts, 0, nbk * sizeof(unsigned long long), st));
     wd::slice_hist_kernel<<<t->sm_count * 4, wd::kBlock, 0, st>>>(io.keys + off, cnt, nbk, s.hseed, counts);
     wd::slice_scan_kernel<<<1, 32, 0, st>>>(counts, nbk, bounds, cursor);
@@ -580,8 +623,11 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
         io.keys + off, io.vals + off, cnt, dst, cursor, nullptr, nbk, s.hseed, 0, cnt, s.counters);
     CK(cudaGetLastError());
     t->launches += 3;
+    ph_end(t, pg);
+    const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, st);
     for (int j = 0; j < nbk; ++j)
       TRY(launch_probe<true>(t, s, wd::InBucket{s.sl_buf, bounds, j}, wd::OutNone{}, cnt, st));
+    ph_end(t, pp);
   }
   CK(cudaEventRecord(s.sl_done, st));
   s.sl_used = true;
@@ -597,7 +643,10 @@ wd_status_t single_op(wd_table* t, int op, const IO& io, cudaStream_t stream) {
     const int nbk = choose_slices(t, s, op, io.n);
     if (nbk > 1) return slice_insert(t, s, io, nbk, stream);
     const wd::InSoA in{io.keys, io.vals, io.n};
-    return probe_soa(t, s, op, in, io.vout, io.fout, io.n, stream);
+    const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, stream);
+    TRY(probe_soa(t, s, op, in, io.vout, io.fout, io.n, stream));
+    ph_end(t, pp);
+    return WD_OK;
   }
   // out-of-core pipeline (Fig. 5): H2D(b+1) || probe(b) || D2H(b-1).  Default
   // batch here 2^22 (not P:197's 2^24): shorter pipeline fill and drain; the bench's e2e
@@ -612,12 +661,14 @@ wd_status_t single_op(wd_table* t, int op, const IO& io, cudaStream_t stream) {
     const int slot = int(b % kStage);
     const uint64_t off = b * B, cnt = std::min(B, io.n - off);
     const uint32_t *dk, *dv;
-    TRY(stage_in(s, io, off, cnt, slot, insert, &dk, &dv));
+    TRY(stage_in(t, s, io, off, cnt, slot, insert, &dk, &dv));
     const wd::InSoA in{dk, dv, cnt};
     uint32_t* ov = nullptr; uint8_t* of = nullptr;
     if (!insert) out_ptrs(s, io, off, slot, &ov, &of);
+    const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, s.s_main);
     TRY(probe_soa(t, s, op, in, ov, of, cnt, s.s_main));
-    TRY(stage_out(s, io, off, cnt, slot, !insert));
+    ph_end(t, pp);
+    TRY(stage_out(t, s, io, off, cnt, slot, !insert));
   }
   return join_into(t, stream, ev0);
 }
@@ -812,6 +863,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
     return WD_OK;
   };
   auto phaseA = [&](uint64_t b) -> wd_status_t {
+    Nvtx nv("wd:A multisplit");
     const unsigned long long e = e0 + 1 + b;
     const int slot = int(e & 1);
     for (size_t r = 0; r < t->local.size(); ++r) {
@@ -820,10 +872,14 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       DeviceGuard g(s.device);
       const uint64_t off = std::min(io.n, b * B), cnt = std::min(B, io.n - off);
       const uint32_t *dk = nullptr, *dv = nullptr;
-      TRY(stage_in(s, io, off, cnt, int(b % kStage), insert, &dk, &dv));
+      TRY(stage_in(t, s, io, off, cnt, int(b % kStage), insert, &dk, &dv));
       if (X == 0 && e > 2) TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e - 2));  // owners released e-2
-      if (cnt) TRY(multisplit(s, dk, dv, cnt, slot));
-      if (insert) TRY(stage_out(s, io, off, cnt, int(b % kStage), false));  // input slot free
+      if (cnt) {
+        const Ph pm = ph_begin(t, wd::PH_MULTISPLIT, s.device, s.s_main);
+        TRY(multisplit(s, dk, dv, cnt, slot));
+        ph_end(t, pm);
+      }
+      if (insert) TRY(stage_out(t, s, io, off, cnt, int(b % kStage), false));  // input slot free
       if (X == 0) {
         TRY(publish(s, slot, e));
       } else {                          // this shard's row of T to the host
@@ -838,6 +894,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
   // flags; NCCL all-gathers T (rank mode), then one grouped send/recv per peer (an
   // all-to-all(v)).  The host waits for this batch's row(s) of T first.
   auto phaseT = [&](uint64_t b) -> wd_status_t {
+    Nvtx nv("wd:T transposition");
     const unsigned long long e = e0 + 1 + b;
     const int slot = int(e & 1);
     for (auto& s : t->local) {
@@ -848,6 +905,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       for (auto& s : t->local) {
         DeviceGuard g(s.device);
         if (e > 2) TRY(launch_wait(t, s, s.s_main, FLAG_DONE, e - 2));   // owners released e-2
+        const Ph px = ph_begin(t, wd::PH_EXCHANGE, s.device, s.s_main);
         for (int d = 0; d < m; ++d) {
           const uint64_t c = std::min<uint64_t>(s.hrow[slot][d], B);
           if (c)
@@ -855,6 +913,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
                                static_cast<char*>(s.send) + uint64_t(d) * B * isz, c * isz,
                                cudaMemcpyDefault, s.s_main));
         }
+        ph_end(t, px);
         TRY(publish(s, slot, e));       // counts + READY after the copies (stream order)
       }
       return WD_OK;
@@ -875,6 +934,11 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       DeviceGuard g(s.device);
       if (s.pdone_rec[slot]) CK(cudaStreamWaitEvent(s.s_main, s.ev_pdone[slot], 0));
     }
+    std::vector<Ph> px;
+    for (auto& s : t->local) {
+      DeviceGuard g(s.device);
+      px.push_back(ph_begin(t, wd::PH_EXCHANGE, s.device, s.s_main));
+    }
     NK(g_nccl.GroupStart());
     for (auto& s : t->local) {
       DeviceGuard g(s.device);
@@ -888,6 +952,10 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       }
     }
     NK(g_nccl.GroupEnd());
+    for (size_t r = 0; r < t->local.size(); ++r) {
+      DeviceGuard g(t->local[r].device);
+      ph_end(t, px[r]);
+    }
     for (auto& s : t->local) {          // my column of T -> recv_count (InSeg), cursor reset
       DeviceGuard g(s.device);
       for (int d = 0; d < m; ++d) s.hcol[slot][d] = T[size_t(d) * m + s.id];
@@ -898,20 +966,22 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
     return WD_OK;
   };
   auto phaseB = [&](uint64_t b) -> wd_status_t {
+    Nvtx nv("wd:B probe");
     const unsigned long long e = e0 + 1 + b;
     const int slot = int(e & 1);
     for (auto& s : t->local) {
       DeviceGuard g(s.device);
       if (X == 2) CK(cudaStreamWaitEvent(s.s_probe, s.ev_ready[slot], 0));
       else TRY(launch_wait(t, s, s.s_probe, FLAG_READY, e));
+      if (X == 0 && !insert && t->res_used[slot])   // origins consumed this result slot
+        TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
+      const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, s.s_probe);
       if (insert) {
         const wd::InSeg<true> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
         TRY(launch_probe<true>(t, s, in, wd::OutNone{}, B, s.s_probe));
       } else {
         const wd::InSeg<false> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
         if (X == 0) {
-          // origins consumed the results of the previous query epoch that used this slot
-          if (t->res_used[slot]) TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
           // reverse transposition: results go straight to their origins' result
           // slots (region s.id of origin d's slot), coalesced remote stores
           wd::OutPacked out{};
@@ -931,6 +1001,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
             TRY(launch_probe<false>(t, s, in, out, B, s.s_probe));
         }
       }
+      ph_end(t, pp);
       if (X == 2) {
         CK(cudaEventRecord(s.ev_pdone[slot], s.s_probe));   // recv[slot] may be refilled
         s.pdone_rec[slot] = true;
@@ -948,12 +1019,14 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
           CK(cudaEventSynchronize(s.ev_col));
         }
         if (t->res_used[slot]) TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
+        const Ph pr = ph_begin(t, wd::PH_REVERSE, s.device, s.s_probe);
         for (int d = 0; d < m; ++d) {
           const uint64_t c = std::min<uint64_t>(col[d], B);
           if (c)
             CK(cudaMemcpyAsync(t->peers[d].res[slot] + uint64_t(s.id) * B,
                                s.res_stage + uint64_t(d) * B, c * 8, cudaMemcpyDefault, s.s_probe));
         }
+        ph_end(t, pr);
       }
     }
     if (!insert && X == 2) {            // reverse transposition with NCCL
@@ -961,6 +1034,11 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       for (auto& s : t->local) {        // own result slot free: own unpermute of e-2
         DeviceGuard g(s.device);
         if (s.unperm_rec[slot]) CK(cudaStreamWaitEvent(s.s_probe, s.ev_unperm[slot], 0));
+      }
+      std::vector<Ph> pr;
+      for (auto& s : t->local) {
+        DeviceGuard g(s.device);
+        pr.push_back(ph_begin(t, wd::PH_REVERSE, s.device, s.s_probe));
       }
       NK(g_nccl.GroupStart());
       for (auto& s : t->local) {
@@ -973,6 +1051,10 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
         }
       }
       NK(g_nccl.GroupEnd());
+      for (size_t r = 0; r < t->local.size(); ++r) {
+        DeviceGuard g(t->local[r].device);
+        ph_end(t, pr[r]);
+      }
     }
     for (auto& s : t->local) {
       DeviceGuard g(s.device);
@@ -983,6 +1065,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
     return WD_OK;
   };
   auto phaseC = [&](uint64_t b) -> wd_status_t {
+    Nvtx nv("wd:C unpermute");
     const unsigned long long e = e0 + 1 + b;
     const int slot = int(e & 1);
     for (size_t r = 0; r < t->local.size(); ++r) {
@@ -999,8 +1082,10 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
         out_ptrs(s, io, off, int(b % kStage), &ov, &of);
         const int grid = int(std::min<uint64_t>((cnt + wd::kBlock - 1) / wd::kBlock,
                                                 uint64_t(t->sm_count) * 8));
+        const Ph pu = ph_begin(t, wd::PH_UNPERMUTE, s.device, s.s_main);
         wd::unpermute_kernel<<<grid, wd::kBlock, 0, s.s_main>>>(s.pos[slot], cnt, src, ov, of);
         CK(cudaGetLastError());
+        ph_end(t, pu);
         t->launches++;
       }
       if (X == 2) {
@@ -1009,7 +1094,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       } else {
         TRY(launch_signal(t, s, s.s_main, FLAG_RESC, e));
       }
-      TRY(stage_out(s, io, off, cnt, int(b % kStage), true));
+      TRY(stage_out(t, s, io, off, cnt, int(b % kStage), true));
     }
     return WD_OK;
   };
@@ -1097,9 +1182,14 @@ void pick_group_size(wd_table* t, int op, uint64_t n) {
   if (op == OP_INSERT) t->est_size = std::min<uint64_t>(t->est_size + n, wd_capacity(t));
 }
 
+const char* op_name(int op) {
+  return op == OP_INSERT ? "wd_insert" : op == OP_RETRIEVE ? "wd_retrieve" : "wd_erase";
+}
+
 wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* vals,
                   uint32_t* vout, uint8_t* fout, uint64_t n, cudaStream_t stream) {
   if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  Nvtx nv(op_name(op));
   IO io;
   io.keys = keys; io.vals = vals; io.vout = vout; io.fout = fout; io.n = n;
   TRY(classify_io(t, op == OP_INSERT, io, -1));
@@ -1119,6 +1209,7 @@ wd_status_t do_op_sharded(wd_table* t, int op, const uint32_t* const* keys,
                           const uint32_t* const* vals, uint32_t* const* vout, uint8_t* const* fout,
                           const uint64_t* n, const wd_stream_t* streams) {
   if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
+  Nvtx nv(op == OP_INSERT ? "wd_insert_sharded" : "wd_retrieve_sharded");
   if (!keys || !n || (op == OP_INSERT && !vals))
     return fail(WD_ERR_INVALID_ARG, "_sharded: NULL array argument");
   const size_t L = t->local.size();
@@ -1380,6 +1471,15 @@ void wd_destroy(wd_table_t* t) {
   }
   for (void* p : t->opened) cudaIpcCloseMemHandle(p);
   if (t->nccl_ready) free_nccl(t);
+  for (auto& kv : t->ph_pool) {
+    DeviceGuard g(kv.first);
+    for (cudaEvent_t e : kv.second) cudaEventDestroy(e);
+  }
+  for (auto& r : t->ph_recs) {
+    DeviceGuard g(r.device);
+    cudaEventDestroy(r.a);
+    cudaEventDestroy(r.b);
+  }
   for (auto& s : t->local) free_staged(s);
   for (auto& s : t->local) shard_free(s);
   if (t->loop_stream) cudaStreamDestroy(t->loop_stream);
@@ -1584,6 +1684,9 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       if (v < 0 || v > wd::kMaxShards) return fail(WD_ERR_INVALID_ARG, "slices %lld", (long long)v);
       t->slices = int(v);
       return WD_OK;
+    case WD_OPT_PHASE_TIMING:
+      t->phase_on = v != 0;
+      return WD_OK;
     case WD_OPT_EXCHANGE:
       if (v < 0 || v > 2) return fail(WD_ERR_INVALID_ARG, "exchange %lld", (long long)v);
       if (v == 2 && t->mode == MODE_LOOPBACK)
@@ -1615,6 +1718,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_SPAN: return t->span;
     case WD_OPT_SLICES: return t->slices;
     case WD_OPT_EXCHANGE: return t->exchange;
+    case WD_OPT_PHASE_TIMING: return t->phase_on ? 1 : 0;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;
     case WD_OPT_LOCAL_SHARDS: return int64_t(t->local.size());
@@ -1622,6 +1726,32 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
   }
   fail(WD_ERR_INVALID_ARG, "unknown option %d", int(opt));
   return INT64_MIN;
+}
+
+wd_status_t wd_phase_times(wd_table_t* t, double ms_out[WD_N_PHASES], uint64_t count_out[WD_N_PHASES]) {
+  if (!t || !ms_out) return fail(WD_ERR_INVALID_ARG, "wd_phase_times arguments");
+  for (int i = 0; i < WD_N_PHASES; ++i) {
+    ms_out[i] = 0.0;
+    if (count_out) count_out[i] = 0;
+  }
+  wd_status_t st = WD_OK;
+  for (auto& r : t->ph_recs) {
+    DeviceGuard g(r.device);
+    float ms = 0.f;
+    if (st == WD_OK) {
+      const cudaError_t e1 = cudaEventSynchronize(r.b);
+      const cudaError_t e2 = e1 == cudaSuccess ? cudaEventElapsedTime(&ms, r.a, r.b) : e1;
+      if (e2 != cudaSuccess) st = fail(WD_ERR_CUDA, "wd_phase_times: %s", cudaGetErrorString(e2));
+    }
+    if (r.phase >= 0 && r.phase < WD_N_PHASES) {
+      ms_out[r.phase] += ms;
+      if (count_out) count_out[r.phase] += 1;
+    }
+    t->ph_pool[r.device].push_back(r.a);
+    t->ph_pool[r.device].push_back(r.b);
+  }
+  t->ph_recs.clear();
+  return st;
 }
 
 wd_status_t wd_last_error(void) { return g_last; }

@@ -171,6 +171,12 @@ struct wd_table {
   // "asynchronous inter-GPU copies"), 2 staged buffers + NCCL send/recv (all-to-all(v) of
   // exact counts after an all-gather of T; the north star's NCCL path)
   int exchange = 0;
+  // per-phase CUDA-event timing (WD_OPT_PHASE_TIMING, wd_phase_times): begin/end event pairs
+  // recorded on the stream each phase runs on; events are pooled per device
+  bool phase_on = false;
+  struct PhaseRec { int phase, device; cudaEvent_t a, b; };
+  std::vector<PhaseRec> ph_recs;
+  std::unordered_map<int, std::vector<cudaEvent_t>> ph_pool;
   bool nccl_ready = false;
   unsigned char nccl_id[128] = {};           // rank mode: rank 0's ncclUniqueId (wd_rank_connect)
   bool have_nccl_id = false;
