@@ -547,8 +547,19 @@ bool needs_staging(const IO& io) { return io.kin != PK_DEVICE || io.kout != PK_D
 enum Op { OP_INSERT = 0, OP_RETRIEVE = 1, OP_ERASE = 2 };
 
 // the probe kernel of one call on a plain (SoA) input
+// (the probe kernels index one launch's input with 32 bits: device calls of >= 2^32 pairs
+// are launched in pieces of 2^31)
 wd_status_t probe_soa(wd_table* t, Shard& s, int op, const wd::InSoA& in, uint32_t* ov, uint8_t* of,
                       uint64_t n, cudaStream_t st) {
+  constexpr uint64_t kPiece = 1ull << 31;
+  if (n >= (1ull << 32)) {
+    for (uint64_t off = 0; off < n; off += kPiece) {
+      const uint64_t c = std::min(kPiece, n - off);
+      const wd::InSoA p{in.keys + off, in.vals ? in.vals + off : nullptr, c};
+      TRY(probe_soa(t, s, op, p, ov ? ov + off : nullptr, of ? of + off : nullptr, c, st));
+    }
+    return WD_OK;
+  }
   if (op == OP_INSERT) return launch_probe<true>(t, s, in, wd::OutNone{}, n, st);
   if (op == OP_ERASE) return launch_probe<false>(t, s, in, wd::OutErase<wd::OutSoA>{{nullptr, of}}, n, st);
   return launch_probe<false>(t, s, in, wd::OutSoA{ov, of}, n, st);
