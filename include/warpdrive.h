@@ -222,7 +222,8 @@ typedef enum {
                                 tables > 512 MB and calls of >= 2^26 pairs (unless the span
                                 read-ahead applies), else 1 (off);
                                 1: off; 2..32: that many slices.  Uses 8 B of scratch per pair,
-                                at most 2^26 pairs at a time, kept for the table's lifetime
+                                two buffers of at most 2^27 pairs (grouping of the next chunk
+                                overlaps the probing of this one), kept for the table's lifetime
                                 (stream-ordered allocation); in auto mode a failed scratch
                                 allocation falls back to the plain launch. */
     WD_OPT_EXCHANGE = 12,    /* how the transposition of P:117 (a8) and its reverse (a10) move

@@ -251,9 +251,18 @@ void shard_free(Shard& s) {
   if (s.s_d2h) cudaStreamSynchronize(s.s_d2h);
   free_exchange(s);
   free_staging(s);
-  if (s.sl_buf) cudaFree(s.sl_buf);
+  for (int b = 0; b < 2; ++b) {
+    if (s.sl_buf[b]) cudaFree(s.sl_buf[b]);
+    if (s.sl_grouped[b]) cudaEventDestroy(s.sl_grouped[b]);
+    if (s.sl_probed[b]) cudaEventDestroy(s.sl_probed[b]);
+  }
   if (s.sl_meta) cudaFree(s.sl_meta);
   if (s.sl_done) cudaEventDestroy(s.sl_done);
+  if (s.sl_fork) cudaEventDestroy(s.sl_fork);
+  if (s.s_group) {
+    cudaStreamSynchronize(s.s_group);
+    cudaStreamDestroy(s.s_group);
+  }
   if (s.slots) cudaFree(s.slots);
   if (s.counters) cudaFree(s.counters);
   for (int i = 0; i < kStage; ++i) {
@@ -580,7 +589,7 @@ int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
   return 16;
 }
 
-// Slice-grouped bulk insert.  Each chunk of <= 2^26 pairs is grouped by the table slice of
+// Slice-grouped bulk insert.  Each chunk of <= 2^27 pairs is grouped by the table slice of
 // its keys' first region (Line 5: h(k) is monotone in fmix32(k + seed), so slice j of nbk
 // holds the region starts [j nb / nbk, (j + 1) nb / nbk)): a histogram, a scan and the
 // multisplit kernel write the pairs slice by slice into a scratch buffer; then one probe
@@ -591,22 +600,37 @@ int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
 // for the probe launches.  Results are those of one launch: the probing of every key is
 // Fig. 3's; only the order in which the keys of one call are inserted changes (C20: any of
 // a call's duplicate values may win).
+// Round 2: the grouping of chunk c + 1 runs on a side stream while chunk c is probed (two
+// scratch buffers, event-ordered), so only the first chunk's grouping is exposed; chunks of
+// 2^27 (tools/gpu_chunk_sweep.sh, 2^28 pairs: 2^25 / 2^26 / 2^27 / 2^28 -> 17.2 / 18.8 /
+// 19.6 / 19.7 G inserts/s: fewer, longer probe launches; WD_SLICE_CHUNK_LOG2 overrides).
 wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStream_t st) {
-  constexpr uint64_t kChunkPairs = 1ull << 26;
+  static const int chunk_log2 = getenv("WD_SLICE_CHUNK_LOG2") ? atoi(getenv("WD_SLICE_CHUNK_LOG2")) : 27;
+  const uint64_t kChunkPairs = 1ull << chunk_log2;
   const uint64_t cap = std::min<uint64_t>(io.n, kChunkPairs);
-  if (!s.sl_done) CK(cudaEventCreateWithFlags(&s.sl_done, cudaEventDisableTiming));
+  const int nbuf = io.n > kChunkPairs ? 2 : 1;
+  if (!s.sl_done) {
+    CK(cudaEventCreateWithFlags(&s.sl_done, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&s.sl_fork, cudaEventDisableTiming));
+    for (int b = 0; b < 2; ++b) {
+      CK(cudaEventCreateWithFlags(&s.sl_grouped[b], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&s.sl_probed[b], cudaEventDisableTiming));
+    }
+    CK(cudaStreamCreateWithFlags(&s.s_group, cudaStreamNonBlocking));
+  }
   if (s.sl_used) CK(cudaStreamWaitEvent(st, s.sl_done, 0));   // scratch of an earlier call
-  if (s.sl_cap < cap) {
+  for (int b = 0; b < nbuf; ++b) {
+    if (s.sl_cap[b] >= cap) continue;
     // stream-ordered (no device synchronisation): the old scratch is released after its
     // last use (st waits on sl_done above), the new one is allocated in st's order.  The
-    // scratch (8 B per pair, <= 512 MB) is kept for the table's lifetime.
-    if (s.sl_buf) CK(cudaFreeAsync(s.sl_buf, st));
-    s.sl_buf = nullptr;
-    s.sl_cap = 0;
-    const cudaError_t e = cudaMallocAsync(&s.sl_buf, cap * sizeof(unsigned long long), st);
+    // scratch (8 B per pair, <= 2 x 1 GB) is kept for the table's lifetime.
+    if (s.sl_buf[b]) CK(cudaFreeAsync(s.sl_buf[b], st));
+    s.sl_buf[b] = nullptr;
+    s.sl_cap[b] = 0;
+    const cudaError_t e = cudaMallocAsync(&s.sl_buf[b], cap * sizeof(unsigned long long), st);
     if (e != cudaSuccess) {
       cudaGetLastError();
-      s.sl_buf = nullptr;
+      s.sl_buf[b] = nullptr;
       if (t->slices == 0) {        // auto: the optimisation steps back, the call still runs
         const wd::InSoA in{io.keys, io.vals, io.n};
         return probe_soa(t, s, OP_INSERT, in, nullptr, nullptr, io.n, st);
@@ -614,31 +638,53 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
       return fail(e == cudaErrorMemoryAllocation ? WD_ERR_OUT_OF_MEMORY : WD_ERR_CUDA,
                   "slice scratch of %llu pairs: %s", (unsigned long long)cap, cudaGetErrorString(e));
     }
-    s.sl_cap = cap;
+    s.sl_cap[b] = cap;
   }
-  if (!s.sl_meta) CK(cudaMalloc(&s.sl_meta, 97 * sizeof(unsigned long long)));
-  unsigned long long* counts = s.sl_meta;
-  unsigned long long* bounds = s.sl_meta + 32;
-  unsigned long long* cursor = s.sl_meta + 65;
-  wd::DstPtrs dst{};
-  for (int d = 0; d < nbk; ++d) dst.p[d] = s.sl_buf;
+  if (!s.sl_meta) CK(cudaMalloc(&s.sl_meta, 2 * 97 * sizeof(unsigned long long)));
+  // the grouping stream starts after everything st has so far (inputs, scratch allocation)
+  CK(cudaEventRecord(s.sl_fork, st));
+  CK(cudaStreamWaitEvent(s.s_group, s.sl_fork, 0));
   const int ms_grid_cap = t->sm_count * blocks_per_sm(wd::multisplit_kernel<true>);
-  for (uint64_t off = 0; off < io.n; off += kChunkPairs) {
-    const uint64_t cnt = std::min(kChunkPairs, io.n - off);
-    const Ph pg = ph_begin(t, wd::PH_GROUP, s.device, st);
-    CK(cudaMemsetAsync(counts, 0, nbk * sizeof(unsigned long long), st));
-    wd::slice_hist_kernel<<<t->sm_count * 4, wd::kBlock, 0, st>>>(io.keys + off, cnt, nbk, s.hseed, counts);
-    wd::slice_scan_kernel<<<1, 32, 0, st>>>(counts, nbk, bounds, cursor);
+  const uint64_t nchunks = (io.n + kChunkPairs - 1) / kChunkPairs;
+  auto group = [&](uint64_t c) -> wd_status_t {   // on s_group, into buffer c % 2
+    const int b = int(c % 2);
+    const uint64_t off = c * kChunkPairs, cnt = std::min(kChunkPairs, io.n - off);
+    unsigned long long* counts = s.sl_meta + b * 97;
+    unsigned long long* bounds = counts + 32;
+    unsigned long long* cursor = counts + 65;
+    if (c >= 2) CK(cudaStreamWaitEvent(s.s_group, s.sl_probed[b], 0));   // probes of c - 2 done
+    const Ph pg = ph_begin(t, wd::PH_GROUP, s.device, s.s_group);
+    CK(cudaMemsetAsync(counts, 0, nbk * sizeof(unsigned long long), s.s_group));
+    wd::slice_hist_kernel<<<t->sm_count * 4, wd::kBlock, 0, s.s_group>>>(io.keys + off, cnt, nbk, s.hseed, counts);
+    wd::slice_scan_kernel<<<1, 32, 0, s.s_group>>>(counts, nbk, bounds, cursor);
+    wd::DstPtrs dst{};
+    for (int d = 0; d < nbk; ++d) dst.p[d] = s.sl_buf[b];
     const uint64_t tiles = (cnt + wd::kMsTile - 1) / wd::kMsTile;
-    wd::multisplit_kernel<true><<<int(std::min<uint64_t>(tiles, uint64_t(ms_grid_cap))), wd::kBlock, 0, st>>>(
+    wd::multisplit_kernel<true><<<int(std::min<uint64_t>(tiles, uint64_t(ms_grid_cap))), wd::kBlock, 0, s.s_group>>>(
         io.keys + off, io.vals + off, cnt, dst, cursor, nullptr, nbk, s.hseed, 0, cnt, s.counters);
     CK(cudaGetLastError());
     t->launches += 3;
     ph_end(t, pg);
+    CK(cudaEventRecord(s.sl_grouped[b], s.s_group));
+    return WD_OK;
+  };
+  auto probe = [&](uint64_t c) -> wd_status_t {   // on st
+    const int b = int(c % 2);
+    const uint64_t off = c * kChunkPairs, cnt = std::min(kChunkPairs, io.n - off);
+    const unsigned long long* bounds = s.sl_meta + b * 97 + 32;
+    CK(cudaStreamWaitEvent(st, s.sl_grouped[b], 0));
     const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, st);
     for (int j = 0; j < nbk; ++j)
-      TRY(launch_probe<true>(t, s, wd::InBucket{s.sl_buf, bounds, j}, wd::OutNone{}, cnt, st));
+      TRY(launch_probe<true>(t, s, wd::InBucket{s.sl_buf[b], bounds, j, j + 1}, wd::OutNone{},
+                             cnt / nbk + 1, st));
     ph_end(t, pp);
+    CK(cudaEventRecord(s.sl_probed[b], st));
+    return WD_OK;
+  };
+  TRY(group(0));
+  for (uint64_t c = 0; c < nchunks; ++c) {
+    if (c + 1 < nchunks) TRY(group(c + 1));
+    TRY(probe(c));
   }
   CK(cudaEventRecord(s.sl_done, st));
   s.sl_used = true;
@@ -1671,7 +1717,7 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       return WD_OK;
     case WD_OPT_PART_SEED: t->pseed = uint32_t(v); return WD_OK;
     case WD_OPT_SLOTS_PER_LANE:
-      if (v != 0 && v != 1 && v != 2 && v != 4 && v != 8)
+      if (v != 0 && v != 1 && v != 2 && v != 4 && v != 8 && v != 16)
         return fail(WD_ERR_INVALID_ARG, "slots per lane %lld", (long long)v);
       t->spl = int(v);
       return WD_OK;

@@ -82,10 +82,12 @@ struct Shard {
   unsigned long long* counters = nullptr;
   // slice-grouped bulk insert (slice_insert): packed-pair scratch for one chunk, and
   // counts[32] | bounds[33] | cursor[32]; sl_done orders reuse across streams
-  unsigned long long* sl_buf = nullptr;
-  uint64_t sl_cap = 0;
+  unsigned long long* sl_buf[2] = {nullptr, nullptr};   // double buffer: group c+1 || probe c
+  uint64_t sl_cap[2] = {0, 0};
   unsigned long long* sl_meta = nullptr;
-  cudaEvent_t sl_done = nullptr;
+  cudaEvent_t sl_done = nullptr, sl_fork = nullptr;
+  cudaEvent_t sl_grouped[2] = {}, sl_probed[2] = {};
+  cudaStream_t s_group = nullptr;
   bool sl_used = false;
   cudaStream_t s_main = nullptr, s_h2d = nullptr, s_d2h = nullptr;
   cudaStream_t s_probe = nullptr;   // phase B of the cascade (own stream unless loopback)
@@ -270,7 +272,10 @@ wd_status_t launch_gv(wd_table* t, Shard& s, const In& in, const Out& out, uint6
     if (k == KS && choose_span(t, s, G, V) == 2)
       return launch_probe_k<G, V, KS, INSERT, In, Out, 2>(t, s, in, out, n_hint, st);
   }
-  if constexpr (V == 1) {
+  if constexpr (V == 16) {          // one lane reads a whole 128-byte window
+    if (k <= 1) return launch_probe_k<G, 16, 1, INSERT>(t, s, in, out, n_hint, st);
+    return launch_probe_k<G, 16, 2, INSERT>(t, s, in, out, n_hint, st);
+  } else if constexpr (V == 1) {
     if (k == 2) return launch_probe_k<G, 1, 2, INSERT>(t, s, in, out, n_hint, st);
     if (k == 4) return launch_probe_k<G, 1, 4, INSERT>(t, s, in, out, n_hint, st);
     return launch_probe_k<G, 1, 8, INSERT>(t, s, in, out, n_hint, st);
@@ -308,7 +313,7 @@ inline int choose_v(const wd_table* t, const Shard& s, int G, bool insert) {
     else v = G >= 2 ? std::max(1, std::min(G / 2, insert && t->align < 16 ? 4 : 8)) : 1;
     if (G == 2 && t->probe_mode == 0) v = 2;
   }
-  v = std::min(v, std::min(G, 8));
+  v = std::min(v, std::min(G, t->spl == 16 ? 16 : 8));
   return v;
 }
 inline int choose_k(const wd_table* t, const Shard& s, int G, int V, bool insert) {
@@ -321,13 +326,22 @@ inline int choose_k(const wd_table* t, const Shard& s, int G, int V, bool insert
   // 4/4 -> 12.9 / 23.5 (16.7), 2/4 -> 13.7 / 21.9 (16.8).
   (void)insert;
   if (V == 4) return 2;
+  if (V == 16) return 1;
   return 2;
 }
 
 template <int G, bool INSERT, class In, class Out>
 wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
+  // sliced bulk inserts (InBucket) on line-aligned tables: one lane reads the whole 128-B
+  // window (V = 16, K = 1; tools/gpu_vk_sweep.sh: 2^28 pairs 18.8 -> 19.7 G inserts/s, 2^24
+  // 20.5 -> 22.8).  Not for queries from HBM: one lane per 128-B line drops them to 9 G/s.
+  if constexpr (G == 16 && INSERT && std::is_same_v<In, wd::InBucket>)
+    if (t->spl == 0 && t->kif == 0 && t->probe_mode == 0 && t->align == 16)
+      return launch_gv<G, 16, INSERT>(t, s, in, out, n_hint, st, 1);
   const int v = choose_v(t, s, G, INSERT), k = choose_k(t, s, G, v, INSERT);
+  if constexpr (G >= 16)
+    if (v == 16) return launch_gv<G, 16, INSERT>(t, s, in, out, n_hint, st, k);
   if constexpr (G >= 8)
     if (v == 8) return launch_gv<G, 8, INSERT>(t, s, in, out, n_hint, st, k);
   if constexpr (G >= 4)
