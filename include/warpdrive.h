@@ -246,6 +246,15 @@ typedef enum {
                                 Results are identical in all three modes. */
     WD_OPT_PHASE_TIMING = 13, /* 1: record CUDA events around every phase of every call (see
                                 wd_phase_times); 0 (default): off */
+    WD_OPT_TAIL = 14,        /* long probe chains (the probing scheme does not depend on
+                                |g|): a key still probing when it enters region number T is
+                                handed to a second launch that probes with |g| = 32, one window
+                                per region (same regions, same order, same leftmost decisions);
+                                a call ends with its longest chain, so small calls get faster.
+                                0 (default): off — measured on B200, the extra launch costs
+                                more than the shorter chains save (profiles/r02/
+                                tail_launch.md); T >= 1: that threshold.  Uses a 24 MB spill
+                                list per shard (keys beyond 2^20 spills just keep probing). */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -169,6 +169,17 @@ void l2_fetch_release(int device) {
   h.set = false;
 }
 
+// ------------------------------------------------------------------ long-chain spill list
+wd_status_t tail_prepare(wd_table* t, Shard& s, cudaStream_t st) {
+  (void)t;
+  if (!s.tail) {
+    CK(cudaMalloc(&s.tail, size_t(kTailCap) * sizeof(wd::TailEntry)));
+    CK(cudaMalloc(&s.tail_count, sizeof(unsigned long long)));
+  }
+  CK(cudaMemsetAsync(s.tail_count, 0, sizeof(unsigned long long), st));
+  return WD_OK;
+}
+
 // ------------------------------------------------------------------ shard lifetime
 wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
                        cudaStream_t shared_main) {
@@ -265,6 +276,8 @@ void shard_free(Shard& s) {
   }
   if (s.slots) cudaFree(s.slots);
   if (s.counters) cudaFree(s.counters);
+  if (s.tail) cudaFree(s.tail);
+  if (s.tail_count) cudaFree(s.tail_count);
   for (int i = 0; i < kStage; ++i) {
     if (s.ev_h2d[i]) cudaEventDestroy(s.ev_h2d[i]);
     if (s.ev_free[i]) cudaEventDestroy(s.ev_free[i]);
@@ -1744,6 +1757,10 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
     case WD_OPT_PHASE_TIMING:
       t->phase_on = v != 0;
       return WD_OK;
+    case WD_OPT_TAIL:
+      if (v < 0 || v > 1000) return fail(WD_ERR_INVALID_ARG, "tail %lld", (long long)v);
+      t->tail = int(v);
+      return WD_OK;
     case WD_OPT_EXCHANGE:
       if (v < 0 || v > 2) return fail(WD_ERR_INVALID_ARG, "exchange %lld", (long long)v);
       if (v == 2 && t->mode == MODE_LOOPBACK)
@@ -1776,6 +1793,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_SLICES: return t->slices;
     case WD_OPT_EXCHANGE: return t->exchange;
     case WD_OPT_PHASE_TIMING: return t->phase_on ? 1 : 0;
+    case WD_OPT_TAIL: return t->tail;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;
     case WD_OPT_LOCAL_SHARDS: return int64_t(t->local.size());

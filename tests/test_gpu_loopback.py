@@ -191,3 +191,19 @@ def test_loopback_rejects_nccl_exchange(wd):
         assert ei.value.status == wd.WD_ERR_UNSUPPORTED
         with pytest.raises(wd.WarpDriveError):
             t.set_option(wd.WD_OPT_EXCHANGE, 3)
+
+
+@pytest.mark.parametrize("exchange", [0, 1])
+def test_loopback_tail_launch(wd, exchange):
+    # the wide tail launch inside the cascade: its answers go through the same reverse
+    # transposition (OutPacked / OutLocalPacked) as the main launch's
+    n = 120_007
+    keys, vals = wdgen.unique_keys(n, 141), wdgen.values(n, 142)
+    q = wdgen.interleaved_queries(n, 141)
+    with wd.Table(capacity_for(n, 0.99), group_size=4, loopback_shards=3, exchange=exchange) as t:
+        t.set_option(wd.WD_OPT_TAIL, 1)
+        t.set_option(wd.WD_OPT_BATCH, 30_000)
+        gv, gf = gpu_roundtrip(t, keys, vals, q)
+        assert t.sync() == 0 and t.size() == n
+    cv, cf = oracle.expected_unique(q, n, 141, 142)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)

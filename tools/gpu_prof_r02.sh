@@ -6,7 +6,7 @@ cd $GRAFT_REPO_ROOT
 TAG=$1; shift
 O=gpurun_out/prof_$TAG
 mkdir -p $O
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:probe_kernel -s 62 -c 3 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:probe_ -s 62 -c 3 \
   -o $O/full python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu "$@" > $O/ncu.log 2>&1
 ncu -i $O/full.ncu-rep --page raw --csv > $O/raw.csv 2>/dev/null
 ncu -i $O/full.ncu-rep --page details --csv > $O/details.csv 2>/dev/null

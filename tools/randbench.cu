@@ -5,10 +5,13 @@
 //   read : window read only (a query)
 //   cas  : window read, then a 64-bit CAS on the window's first slot that FAILS (no write)
 //   casw : ... a CAS that SUCCEEDS (dirty sector, written back later: an insert)
-// Reports windows/s and useful GB/s for 2.26 GB (config 2 table) and 36 GB buffers.
+// Reports windows/s and useful GB/s for the buffer sizes given (GB; default 2.26 = config 2's
+// table and 36 = config 3's; 0.0088 = config 1's L2-resident table).
 // Build: nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o tools/randbench tools/randbench.cu
 #include <cstdio>
 #include <cstdint>
+#include <cstdlib>
+#include <vector>
 #include <cuda_runtime.h>
 
 __device__ __forceinline__ uint32_t hash32(uint32_t x) {
@@ -187,11 +190,16 @@ void run(const char* name, unsigned long long* buf, uint64_t bytes, int grid, in
          WB, AB, D, windows / (ms * 1e-3) / 1e9, windows * WB / (ms * 1e-3) / 1e9);
 }
 
-int main() {
+int main(int argc, char** argv) {
   int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
   unsigned long long* sink; cudaMalloc(&sink, 8);
   cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, 32);
-  for (double gb : {2.26, 36.0}) {
+  // buffer sizes in GB from the command line (default: the config-2 table and config 3);
+  // 0.0088 = config 1's 8.8 MB table, L2-resident: its ceiling is the L2's random rate
+  std::vector<double> sizes;
+  for (int i = 1; i < argc; ++i) sizes.push_back(atof(argv[i]));
+  if (sizes.empty()) sizes = {2.26, 36.0};
+  for (double gb : sizes) {
     const uint64_t bytes = uint64_t(gb * 1e9) / 256 * 256;
     unsigned long long* buf;
     if (cudaMalloc(&buf, bytes) != cudaSuccess) { printf("alloc %.1f GB failed\n", gb); continue; }

@@ -19,7 +19,7 @@ import paper_conf_ipps_junger0s18_b200 as wd  # noqa: E402
 import wdgen.gpu as gg  # noqa: E402
 
 OPT = {"slices": wd.WD_OPT_SLICES, "v": wd.WD_OPT_SLOTS_PER_LANE, "k": wd.WD_OPT_KEYS_IN_FLIGHT,
-       "span": wd.WD_OPT_SPAN, "mode": wd.WD_OPT_PROBE_MODE}
+       "span": wd.WD_OPT_SPAN, "mode": wd.WD_OPT_PROBE_MODE, "tail": wd.WD_OPT_TAIL}
 
 
 def main():
@@ -27,10 +27,13 @@ def main():
     alpha = float(sys.argv[3]) if len(sys.argv) > 3 and "=" not in sys.argv[3] else 0.95
     kv = dict(a.split("=") for a in sys.argv[3:] if "=" in a)
     reps = int(kv.pop("reps", 5))
+    inter = kv.pop("q", "") == "inter"      # config 1: all keys + as many absent, interleaved
     n = 1 << lg
     keys, vals = gg.unique_keys(n, 11), gg.values(n, 12)
-    vo = torch.empty(n, dtype=torch.int32, device="cuda")
-    fo = torch.empty(n, dtype=torch.uint8, device="cuda")
+    qk = gg.interleaved_queries(n, 11) if inter else keys
+    nq = qk.numel()
+    vo = torch.empty(nq, dtype=torch.int32, device="cuda")
+    fo = torch.empty(nq, dtype=torch.uint8, device="cuda")
     s = torch.cuda.current_stream()
     with wd.Table(int(math.ceil(n / alpha)), 1, G) as t:
         for k, v in kv.items():
@@ -42,21 +45,30 @@ def main():
             a.record(s)
             t.insert(keys, vals, s)
             b.record(s)
-            t.retrieve(keys, vo, fo, s)
+            t.retrieve(qk, vo, fo, s)
             c.record(s)
             torch.cuda.synchronize()
             if r:
                 ti.append(a.elapsed_time(b))
                 tq.append(b.elapsed_time(c))
         assert t.sync() == 0 and t.size() == n
-        bad, first, found = gg.check_unique(keys, vo, fo, n, 11, 12)
+        t.phase_times()
+        t.set_option(wd.WD_OPT_PHASE_TIMING, 1)
+        t.clear(s)
+        t.insert(keys, vals, s)
+        ph_ins = {k: round(v[0], 4) for k, v in t.phase_times().items() if v[1]}
+        t.retrieve(qk, vo, fo, s)
+        ph_q = {k: round(v[0], 4) for k, v in t.phase_times().items() if v[1]}
+        t.set_option(wd.WD_OPT_PHASE_TIMING, 0)
+        bad, first, found = gg.check_unique(qk, vo, fo, n, 11, 12)
         assert bad == 0 and found == n
         ims, qms = sum(ti) / len(ti), sum(tq) / len(tq)
         print(json.dumps({"n_log2": lg, "G": G, "alpha": alpha, "opts": kv,
-                          "kernel": os.environ.get("WD_PROBE_KERNEL", "lean"),
+                          "env": {k: v for k, v in os.environ.items() if k.startswith("WD_")},
                           "table_MB": t.capacity() * 8 / 1e6,
-                          "insert_gops": n / ims / 1e6, "query_gops": n / qms / 1e6,
-                          "insert_ms": ims, "query_ms": qms}), flush=True)
+                          "insert_gops": n / ims / 1e6, "query_gops": nq / qms / 1e6, "queries": nq,
+                          "insert_ms": ims, "query_ms": qms, "insert_phases_ms": ph_ins,
+                          "query_phases_ms": ph_q}), flush=True)
 
 
 if __name__ == "__main__":
