@@ -19,7 +19,8 @@ import paper_conf_ipps_junger0s18_b200 as wd  # noqa: E402
 import wdgen.gpu as gg  # noqa: E402
 
 OPT = {"slices": wd.WD_OPT_SLICES, "v": wd.WD_OPT_SLOTS_PER_LANE, "k": wd.WD_OPT_KEYS_IN_FLIGHT,
-       "span": wd.WD_OPT_SPAN, "mode": wd.WD_OPT_PROBE_MODE, "tail": wd.WD_OPT_TAIL}
+       "span": wd.WD_OPT_SPAN, "mode": wd.WD_OPT_PROBE_MODE, "tail": wd.WD_OPT_TAIL,
+       "flags": wd.WD_OPT_KERNEL_FLAGS}
 
 
 def main():
@@ -27,10 +28,11 @@ def main():
     alpha = float(sys.argv[3]) if len(sys.argv) > 3 and "=" not in sys.argv[3] else 0.95
     kv = dict(a.split("=") for a in sys.argv[3:] if "=" in a)
     reps = int(kv.pop("reps", 5))
-    inter = kv.pop("q", "") == "inter"      # config 1: all keys + as many absent, interleaved
+    qmode = kv.pop("q", "")                 # inter: config 1 (all keys + as many absent,
+    inter = qmode == "inter"                # interleaved); miss: absent keys only
     n = 1 << lg
     keys, vals = gg.unique_keys(n, 11), gg.values(n, 12)
-    qk = gg.interleaved_queries(n, 11) if inter else keys
+    qk = gg.interleaved_queries(n, 11) if inter else (gg.unique_keys(n, 11, start=n) if qmode == "miss" else keys)
     nq = qk.numel()
     vo = torch.empty(nq, dtype=torch.int32, device="cuda")
     fo = torch.empty(nq, dtype=torch.uint8, device="cuda")
@@ -61,7 +63,7 @@ def main():
         ph_q = {k: round(v[0], 4) for k, v in t.phase_times().items() if v[1]}
         t.set_option(wd.WD_OPT_PHASE_TIMING, 0)
         bad, first, found = gg.check_unique(qk, vo, fo, n, 11, 12)
-        assert bad == 0 and found == n
+        assert bad == 0 and found == (0 if qmode == "miss" else n)
         ims, qms = sum(ti) / len(ti), sum(tq) / len(tq)
         print(json.dumps({"n_log2": lg, "G": G, "alpha": alpha, "opts": kv,
                           "env": {k: v for k, v in os.environ.items() if k.startswith("WD_")},
