@@ -218,11 +218,13 @@ typedef enum {
     WD_OPT_SLICES = 11,      /* a bulk insert of device-resident pairs into a single-shard table
                                 is grouped by table slice of the keys' first region (Line 5) and
                                 inserted with one probe launch per slice (better L2 reuse); the
-                                probing of each key is unchanged.  0 (default): 16 slices for
-                                tables > 512 MB and calls of >= 2^26 pairs (unless the span
-                                read-ahead applies), else 1 (off);
+                                probing of each key is unchanged.  0 (default): for tables > 512 MB
+                                and calls of >= 2^26 pairs (unless the span read-ahead
+                                applies), the power of two that makes a slice <= 160 MB
+                                (16 for config 2's 2.3 GB), at most 32, and off when a slice
+                                would exceed 300 MB (measured slower);
                                 1: off; 2..32: that many slices.  Uses 8 B of scratch per pair,
-                                two buffers of at most 2^27 pairs (grouping of the next chunk
+                                two buffers of at most 2^28 pairs (grouping of the next chunk
                                 overlaps the probing of this one), kept for the table's lifetime
                                 (stream-ordered allocation); in auto mode a failed scratch
                                 allocation falls back to the plain launch. */
@@ -291,6 +293,13 @@ wd_status_t wd_phase_times(wd_table_t* t, double ms_out[WD_N_PHASES], uint64_t c
 wd_status_t wd_last_error(void);
 const char* wd_error_string(wd_status_t s);
 const char* wd_last_error_message(void);
+
+/* Probe accounting under concurrency (SURVEY §8(d) "replaced by the measured values from the
+ * WD_COUNT_PROBES build"): windows examined, distinct 128-byte lines touched, CAS attempts,
+ * CAS lost to a concurrent insert, keys probed — summed since the last call over the probe
+ * launches of local shard `shard`, then reset.  Synchronizes.  WD_ERR_UNSUPPORTED unless the
+ * library was built with -DWD_COUNT_PROBES (a measurement build: tools/probe_counts.py). */
+wd_status_t wd_probe_counts(wd_table_t* t, int shard, uint64_t out[5]);
 
 /* slots of local shard `shard` (0-based among this process's shards) */
 uint64_t    wd_shard_capacity(wd_table_t* t, int shard);

@@ -48,7 +48,8 @@ EXPORTS = ["wd_create", "wd_create_loopback", "wd_create_rank", "wd_rank_handle"
            "wd_destroy", "wd_clear", "wd_insert", "wd_retrieve", "wd_size", "wd_capacity",
            "wd_sync", "wd_set_option", "wd_get_option", "wd_last_error", "wd_error_string",
            "wd_last_error_message", "wd_shard_capacity", "wd_dump", "wd_counters", "wd_erase",
-           "wd_rebuild", "wd_insert_sharded", "wd_retrieve_sharded", "wd_phase_times"]
+           "wd_rebuild", "wd_insert_sharded", "wd_retrieve_sharded", "wd_phase_times",
+           "wd_probe_counts"]
 
 
 class WarpDriveError(RuntimeError):
@@ -96,6 +97,7 @@ def _load():
         "wd_insert_sharded": ([p, p, p, p, p], i32),
         "wd_retrieve_sharded": ([p, p, p, p, p, p], i32),
         "wd_phase_times": ([p, p, p], i32),
+        "wd_probe_counts": ([p, i32, p], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -337,6 +339,13 @@ class Table:
         cnt = (C.c_uint64 * len(PHASES))()
         _check(_lib.wd_phase_times(self._h, C.addressof(ms), C.addressof(cnt)))
         return {p: (ms[i], int(cnt[i])) for i, p in enumerate(PHASES)}
+
+    def probe_counts(self, shard: int = 0) -> dict:
+        """Windows / 128-B lines / CAS attempts / CAS lost / keys of the probe launches since
+        the last call (a -DWD_COUNT_PROBES build only; else WarpDriveError UNSUPPORTED)."""
+        out = np.zeros(5, np.uint64)
+        _check(_lib.wd_probe_counts(self._h, shard, out.ctypes.data))
+        return dict(zip(("windows", "lines", "cas", "cas_lost", "keys"), (int(x) for x in out)))
 
     @property
     def launches(self) -> int:

@@ -592,17 +592,25 @@ wd_status_t probe_soa(wd_table* t, Shard& s, int op, const wd::InSoA& in, uint32
 // Auto only where it was measured to pay (profiles/r01_slices.txt: 2^28 pairs into 2.3 GB;
 // 16 slices over 2^24-pair chunks were SLOWER than one launch): calls of >= 2^26 pairs, so
 // each slice launch gets >= 2^22 keys, and not where the plain launch uses the span
-// read-ahead (|g| = 1), whose gain the sliced launches (InBucket) do not have.
+// read-ahead (|g| = 1), whose gain the sliced launches (InBucket) do not have.  The slice
+// count follows the table: slices of ~128-280 MB pay, slices of ~540 MB are SLOWER than no
+// slicing (profiles/r02/capacity_knee.md, 2^29 pairs at alpha 0.5 into 8.6 GB: 16 slices
+// 9.9, none 17.1, 32 slices 22.1 G inserts/s); at most 32 slices, so tables above ~9.6 GB
+// are not sliced.
 int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
   if (op != OP_INSERT || t->serial || t->slices == 1) return 1;
   if (t->slices > 1) return t->slices;
-  if (s.cap * sizeof(unsigned long long) <= (512ull << 20) || n < (1ull << 26)) return 1;
+  const double tb = double(s.cap) * sizeof(unsigned long long);
+  if (tb <= double(512ull << 20) || n < (1ull << 26)) return 1;
   const int v = choose_v(t, s, t->G_used, true);
   if (choose_span(t, s, t->G_used, v) == 2) return 1;
-  return 16;
+  int nbk = 2;
+  while (nbk < wd::kMaxShards && tb / nbk > 160e6) nbk *= 2;
+  if (tb / nbk > 300e6) return 1;
+  return nbk;
 }
 
-// Slice-grouped bulk insert.  Each chunk of <= 2^27 pairs is grouped by the table slice of
+// Slice-grouped bulk insert.  Each chunk of <= 2^28 pairs is grouped by the table slice of
 // its keys' first region (Line 5: h(k) is monotone in fmix32(k + seed), so slice j of nbk
 // holds the region starts [j nb / nbk, (j + 1) nb / nbk)): a histogram, a scan and the
 // multisplit kernel write the pairs slice by slice into a scratch buffer; then one probe
@@ -615,10 +623,11 @@ int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
 // a call's duplicate values may win).
 // Round 2: the grouping of chunk c + 1 runs on a side stream while chunk c is probed (two
 // scratch buffers, event-ordered), so only the first chunk's grouping is exposed; chunks of
-// 2^27 (tools/gpu_chunk_sweep.sh, 2^28 pairs: 2^25 / 2^26 / 2^27 / 2^28 -> 17.2 / 18.8 /
-// 19.6 / 19.7 G inserts/s: fewer, longer probe launches; WD_SLICE_CHUNK_LOG2 overrides).
+// 2^28 (tools/gpu_chunk_sweep.sh, 2^28 pairs: 2^25 / 2^26 / 2^27 / 2^28 -> 17.2 / 18.8 /
+// 19.6 / 19.7 G inserts/s; 2^29 pairs into 8.6 GB: 2^27 / 2^28 / 2^29 -> 21.2 / 22.1 / 22.6:
+// fewer, longer probe launches; WD_SLICE_CHUNK_LOG2 overrides).
 wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStream_t st) {
-  static const int chunk_log2 = getenv("WD_SLICE_CHUNK_LOG2") ? atoi(getenv("WD_SLICE_CHUNK_LOG2")) : 27;
+  static const int chunk_log2 = getenv("WD_SLICE_CHUNK_LOG2") ? atoi(getenv("WD_SLICE_CHUNK_LOG2")) : 28;
   const uint64_t kChunkPairs = 1ull << chunk_log2;
   const uint64_t cap = std::min<uint64_t>(io.n, kChunkPairs);
   const int nbuf = io.n > kChunkPairs ? 2 : 1;
@@ -636,7 +645,7 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
     if (s.sl_cap[b] >= cap) continue;
     // stream-ordered (no device synchronisation): the old scratch is released after its
     // last use (st waits on sl_done above), the new one is allocated in st's order.  The
-    // scratch (8 B per pair, <= 2 x 1 GB) is kept for the table's lifetime.
+    // scratch (8 B per pair, <= 2 x 2 GB) is kept for the table's lifetime.
     if (s.sl_buf[b]) CK(cudaFreeAsync(s.sl_buf[b], st));
     s.sl_buf[b] = nullptr;
     s.sl_cap[b] = 0;
@@ -1829,6 +1838,21 @@ wd_status_t wd_phase_times(wd_table_t* t, double ms_out[WD_N_PHASES], uint64_t c
   return st;
 }
 
+wd_status_t wd_probe_counts(wd_table_t* t, int shard, uint64_t out[5]) {
+  if (!t || shard < 0 || shard >= int(t->local.size()) || !out)
+    return fail(WD_ERR_INVALID_ARG, "wd_probe_counts arguments");
+#ifndef WD_COUNT_PROBES
+  return fail(WD_ERR_UNSUPPORTED, "probe accounting needs a -DWD_COUNT_PROBES build of the library");
+#else
+  Shard& s = t->local[shard];
+  DeviceGuard g(s.device);
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpy(out, s.counters + wd::CNT_WIN, 5 * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemset(s.counters + wd::CNT_WIN, 0, 5 * 8));
+  return WD_OK;
+#endif
+}
+
 wd_status_t wd_last_error(void) { return g_last; }
 
 const char* wd_error_string(wd_status_t s) {
@@ -1869,7 +1893,7 @@ wd_status_t wd_counters(wd_table_t* t, int shard, uint64_t out[6]) {
   Shard& s = t->local[shard];
   DeviceGuard g(s.device);
   CK(cudaDeviceSynchronize());
-  CK(cudaMemcpy(out, s.counters, wd::CNT_N * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(out, s.counters, 6 * 8, cudaMemcpyDeviceToHost));   // the ABI's six (probe counts: wd_probe_counts)
   return WD_OK;
 }
 
