@@ -20,7 +20,8 @@ roofline   = the dominant call (CUDA-event time inside the timed region; the ret
              (MEASURED_PEAKS.json), with the ALGORITHMIC bytes of SURVEY §8(d): insert
              8 + 32 S_ins + 32 B, hit query 9 + 32 S_hit B, S from the oracle's sequential
              Fig. 3 replay (tests/golden/probe_cost.json, written by tools/probe_cost.py);
-             `traffic` = measured DRAM bytes per call (profiles/traffic.json, ncu), and
+             `traffic` = measured DRAM bytes of those launches per call (profiles/traffic.json,
+             ncu launch list, tools/traffic_per_call.py), and
              `pattern_ceiling` = the same call against this B200's measured random-access
              rate for the probe's access pattern (profiles/ceilings.json).
 cpu_baseline = the oracle (single-threaded C dictionary) on a bounded sample.
@@ -537,7 +538,7 @@ def run_config(args):
         line["insert_gops"] = nn / (sub[0] * 1e-3) / 1e9
         line["query_gops"] = nn / (sub[1] * 1e-3) / 1e9
         line["nvlink"] = {"insert": _nvlink(world, 8, nn / world, phases.get("multisplit") if args.exchange == 0 else phases.get("exchange")),
-                          "query": _nvlink(world, 12, nn / world, phases.get("probe") if args.exchange == 0 else phases.get("reverse"))}
+                          "query": _nvlink(world, 12, nn / world, phases.get("probe_query") if args.exchange == 0 else phases.get("reverse"))}
     else:
         line["mix"] = {str(h): {"query_gops": q_total / (sub[i] * 1e-3) / 1e9, "ms": sub[i]}
                        for i, h in enumerate((0.0, 0.5, 1.0))}
@@ -638,9 +639,14 @@ def main():
     assert ok, "measured configuration returned wrong results"
 
     # ---- timed region: device-resident
+    # the library brackets every phase (slice grouping, probe launches, ...) with CUDA events
+    # on the stream it runs on (WD_OPT_PHASE_TIMING): the probe kernels' own time over the
+    # timed steps is the roofline's launch time (a few event records per call)
     launches0 = table.launches
     marks = [[ev(), ev(), ev()] for _ in range(args.steps)]
     e0, e1 = ev(), ev()
+    table.phase_times()
+    table.set_option(wd.WD_OPT_PHASE_TIMING, 1)
     with ClockSampler(dev) as clk:
         barrier()
         e0.record(stream)
@@ -649,6 +655,9 @@ def main():
         e1.record(stream)
         barrier()
     launches = table.launches - launches0
+    ph_timed = table.phase_times()
+    table.set_option(wd.WD_OPT_PHASE_TIMING, 0)
+    phases = {k: round(v[0] / args.steps, 4) for k, v in ph_timed.items() if v[1]}
     t_local = e0.elapsed_time(e1) / args.steps
     ins_local = sum(a.elapsed_time(b) for a, b, _ in marks) / args.steps
     qry_local = sum(b.elapsed_time(c) for _, b, c in marks) / args.steps
@@ -659,24 +668,25 @@ def main():
     ops = 2 * n * world
     value = ops / (t_ms * 1e-3) / 1e9
     assert table.sync() == 0
-    # per-phase decomposition (Fig. 11) of one more, instrumented step (not the timed ones)
-    phases = _phases(table, wd, lambda: step())
     nvlink = None
     if world > 1:
         nvlink = {"insert": _nvlink(world, 8, n, phases.get("multisplit") if args.exchange == 0 else phases.get("exchange")),
-                  "query": _nvlink(world, 12, n, phases.get("probe") if args.exchange == 0 else phases.get("reverse"))}
+                  "query": _nvlink(world, 12, n, phases.get("probe_query") if args.exchange == 0 else phases.get("reverse"))}
 
     # ---- roofline of the dominant kernel (single GPU: one launch per call)
     pc = probe_cost(args.alpha, G)
     hbm, peak_src = peaks()
     b_ins = 8 + 32 * pc["ins_sectors"] + 32
     b_hit = 9 + 32 * pc["hit_sectors"]
-    kern = {"insert": (ins_ms, b_ins), "retrieve": (qry_ms, b_hit)}
+    # the probe kernels' own time (all launches of the call), else the call time
+    k_ins = phases.get("probe", ins_ms) if world == 1 else ins_ms
+    k_qry = phases.get("probe_query", qry_ms) if world == 1 else qry_ms
+    kern = {"insert": (k_ins, b_ins, ins_ms), "retrieve": (k_qry, b_hit, qry_ms)}
     dom = max(kern, key=lambda k: kern[k][0])
     other = "retrieve" if dom == "insert" else "insert"
 
     def roof(name):
-        ms, bpo = kern[name]
+        ms, bpo, call_ms = kern[name]
         ach = n * bpo / (ms * 1e-3) / 1e9
         # N > 1: the insert / retrieve call is the whole cascade (multisplit + NVLink push,
         # flags, local probe, reverse pull + unpermute), timed as one call on the stream
@@ -684,15 +694,17 @@ def main():
             kname = (f"{name} cascade a6-a10 over {world} ranks (call time, not one launch; "
                      f"the N=1 line carries the per-kernel roofline)")
         elif per_call[name] == 1:
-            kname = f"probe_kernel<{name}> (G={G})"
+            kname = f"probe_kernel<{name}> (G={G}), one launch per call"
         else:
-            kname = (f"{name} call, {per_call[name]} launches: per 2^26-pair chunk a slice "
-                     f"histogram, a scan, the multisplit and one probe_kernel<{name}> launch "
-                     f"per table slice (WD_OPT_SLICES); call time, algorithmic bytes of the "
-                     f"probe (profiles/r01_launches.csv has the per-launch split)")
+            kname = (f"probe_kernel<{name}, InBucket> (G={G}): the {per_call[name] - 3} probe "
+                     f"launches of the slice-grouped call (one per table slice, WD_OPT_SLICES), "
+                     f"their summed CUDA-event time over the timed steps; the call adds the "
+                     f"slice grouping (histogram, scan, multisplit; `call` below)")
+        call_ach = n * bpo / (call_ms * 1e-3) / 1e9
         return {"kernel": kname, "bound": "hbm", "achieved": ach,
                 "peak": hbm, "unit": "GB/s", "frac": ach / hbm, "traffic": None,
                 "bytes_per_op": bpo, "launch_ms": ms, "launches_per_call": per_call[name],
+                "call": {"ms": call_ms, "achieved": call_ach, "frac": call_ach / hbm},
                 "sectors_per_op": pc["ins_sectors" if name == "insert" else "hit_sectors"],
                 # HBM moves whole 128-B lines for random accesses (C2): the
                 # same kernel against the replay's distinct lines per op
@@ -739,9 +751,12 @@ def main():
     if os.path.exists(traffic_file) and world == 1:
         tj = json.load(open(traffic_file))
         for r, name in ((roofline, dom), (roofline["other"], other)):
-            tr = tj.get(f"{name}_G{G}_a{args.alpha}_n{args.n_log2}")
+            tr = tj.get(f"{name}_probe_G{G}_a{args.alpha}_n{args.n_log2}")
             if tr:
-                r["traffic"] = tr
+                r["traffic"] = tr                       # DRAM bytes of the probe launches
+            trc = tj.get(f"{name}_G{G}_a{args.alpha}_n{args.n_log2}")
+            if trc:
+                r["call"]["traffic"] = trc              # ... of the whole call
 
     # ---- e2e: the same step through the C-ABI with pinned host buffers
     e2e = None

@@ -282,11 +282,13 @@ int64_t     wd_get_option(wd_table_t* t, wd_option_t opt);   /* INT64_MIN on err
 #define WD_PHASE_GROUP 1       /* slice grouping of a bulk insert (histogram, scan, multisplit) */
 #define WD_PHASE_MULTISPLIT 2  /* a6 (fused mode: includes the transposition a8) */
 #define WD_PHASE_EXCHANGE 3    /* a8 staged: copy engine / NCCL send+recv */
-#define WD_PHASE_PROBE 4       /* a3 / a4 / a9 probe kernels (fused mode: includes a10's push) */
+#define WD_PHASE_PROBE 4       /* a3 / a9 insert probe kernels */
 #define WD_PHASE_REVERSE 5     /* a10 staged: results back to their origins */
 #define WD_PHASE_UNPERMUTE 6   /* a10: gather into input order */
 #define WD_PHASE_D2H 7         /* a11: device -> host copies of the results */
-#define WD_N_PHASES 8
+#define WD_PHASE_PROBE_QUERY 8 /* a4 / a9 retrieve / erase probe kernels (fused mode: includes
+                                  a10's push of the answers) */
+#define WD_N_PHASES 9
 wd_status_t wd_phase_times(wd_table_t* t, double ms_out[WD_N_PHASES], uint64_t count_out[WD_N_PHASES]);
 
 /* ------------------------------------------------------------------ diagnostics ---- */

@@ -722,7 +722,7 @@ wd_status_t single_op(wd_table* t, int op, const IO& io, cudaStream_t stream) {
     const int nbk = choose_slices(t, s, op, io.n);
     if (nbk > 1) return slice_insert(t, s, io, nbk, stream);
     const wd::InSoA in{io.keys, io.vals, io.n};
-    const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, stream);
+    const Ph pp = ph_begin(t, op == OP_INSERT ? wd::PH_PROBE : wd::PH_PROBE_QUERY, s.device, stream);
     TRY(probe_soa(t, s, op, in, io.vout, io.fout, io.n, stream));
     ph_end(t, pp);
     return WD_OK;
@@ -744,7 +744,7 @@ wd_status_t single_op(wd_table* t, int op, const IO& io, cudaStream_t stream) {
     const wd::InSoA in{dk, dv, cnt};
     uint32_t* ov = nullptr; uint8_t* of = nullptr;
     if (!insert) out_ptrs(s, io, off, slot, &ov, &of);
-    const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, s.s_main);
+    const Ph pp = ph_begin(t, insert ? wd::PH_PROBE : wd::PH_PROBE_QUERY, s.device, s.s_main);
     TRY(probe_soa(t, s, op, in, ov, of, cnt, s.s_main));
     ph_end(t, pp);
     TRY(stage_out(t, s, io, off, cnt, slot, !insert));
@@ -1054,7 +1054,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       else TRY(launch_wait(t, s, s.s_probe, FLAG_READY, e));
       if (X == 0 && !insert && t->res_used[slot])   // origins consumed this result slot
         TRY(launch_wait(t, s, s.s_probe, FLAG_RESC, t->res_used[slot]));
-      const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, s.s_probe);
+      const Ph pp = ph_begin(t, insert ? wd::PH_PROBE : wd::PH_PROBE_QUERY, s.device, s.s_probe);
       if (insert) {
         const wd::InSeg<true> in{s.self.recv[slot], s.self.recv_count[slot], B, m};
         TRY(launch_probe<true>(t, s, in, wd::OutNone{}, B, s.s_probe));

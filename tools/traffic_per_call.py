@@ -49,6 +49,9 @@ for call in ("insert", "retrieve"):
     b = [sum(m.get("dram__bytes_read.sum", 0) + m.get("dram__bytes_write.sum", 0) for _, m in s[call]) for s in steps]
     t = [sum(m["gpu__time_duration.sum"] for _, m in s[call]) for s in steps]
     out[f"{call}_G{G}_a{alpha}_n{lg}"] = sum(b) / len(b)
+    bp = [sum(m.get("dram__bytes_read.sum", 0) + m.get("dram__bytes_write.sum", 0)
+              for name, m in s[call] if "probe_kernel" in name) for s in steps]
+    out[f"{call}_probe_G{G}_a{alpha}_n{lg}"] = sum(bp) / len(bp)   # the probe launches only
     print(f"{call}: {len(steps)} steps, {sum(len(s[call]) for s in steps) / len(steps):.0f} launches/call, "
           f"{sum(t) / len(t) / 1e6:.2f} ms, {sum(b) / len(b) / 1e9:.2f} GB DRAM per call")
 for s in steps:
