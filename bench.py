@@ -149,10 +149,11 @@ def peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def cpu_baseline_sample(log2n: int = 26):
-    """The oracle as it stands (single-threaded C dictionary), on a bounded sample of the
-    same workload: 2^log2n unique inserts + 2^log2n hit queries (inputs from the same
-    counter-based generator, produced on the device and copied to the host)."""
+def cpu_baseline_sample(log2n: int = 28):
+    """The oracle as it stands (single-threaded C dictionary) on config 2's FULL size by
+    default (2^28 unique inserts + 2^28 hit queries, ~30 s on one core of the
+    GPU box, profiles/r02/oracle_full.json); inputs from the same counter-based generator,
+    produced on the device and copied to the host.  --n-log2 below 28 scales it down."""
     import numpy as np
     import oracle
     n = 1 << log2n
@@ -171,8 +172,8 @@ def cpu_baseline_sample(log2n: int = 26):
     t2 = time.perf_counter()
     assert int(f.sum()) == n and np.array_equal(v, vals)
     return {"value": 2 * n / (t2 - t0) / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"2^{log2n} unique inserts + 2^{log2n} hit queries (config-2 workload, "
-                      f"bounded), single-threaded C dictionary",
+            "sample": f"2^{log2n} unique inserts + 2^{log2n} hit queries (config-2 workload"
+                      f"{', full size' if log2n == 28 else ', scaled'}), single-threaded C dictionary",
             "insert_gops": n / (t1 - t0) / 1e9, "query_gops": n / (t2 - t1) / 1e9,
             "seconds": t2 - t0, "host_cpus": os.cpu_count()}
 
@@ -285,16 +286,23 @@ def run_reference(args):
     times = []
     if args.config in (2, 3):
         keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
-        sample = f"2^22 unique inserts + 2^22 hit queries per step (config-{args.config} keys, generator indices [0, 2^22))"
+        sample = (f"2^22 unique inserts + 2^22 hit queries per step (config-{args.config} keys, generator "
+                  f"indices [0, 2^22){'; the 1/1024 subset of config 3' if args.config == 3 else ''})")
         ops = 2 * n
     elif args.config == 4:
-        keys, vals = wdgen.unique_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
-        qs = [wdgen.mixed_queries(n, 2 * n, h, KEY_SEED)[0] for h in (0.0, 0.5, 1.0)]
-        sample = "2^22-key table (untimed insert) + 3 x 2^23 queries at 0 / 50 / 100 % hits per step"
-        ops = 6 * n
+        # the 1/1024 subset of config 4: a 2^21-key table, 2^22 queries per mix
+        nt = n // 2
+        keys, vals = wdgen.unique_keys(nt, KEY_SEED), wdgen.values(nt, VAL_SEED)
+        qs = [wdgen.mixed_queries(nt, n, h, KEY_SEED)[0] for h in (0.0, 0.5, 1.0)]
+        sample = ("oracle rate on the 1/1024 subset: 2^21-key table (untimed insert) + 3 x 2^22 "
+                  "queries at 0 / 50 / 100 % hits per step")
+        ops = 3 * n
     else:
+        # the 1/1024 subset of config 5's 2^35 draws
+        n = 1 << 25
         keys, vals = wdgen.uniform_keys(n, KEY_SEED), wdgen.values(n, VAL_SEED)
-        sample = "2^22 uniform draws with replacement (duplicate mode) inserted + queried back per step"
+        sample = ("oracle rate on the 1/1024 subset: 2^25 uniform draws with replacement "
+                  "(duplicate mode) inserted + queried back per step")
         ops = 2 * n
     for it in range(args.warmup + args.steps):
         m = oracle.Map(n, dup_mode=args.config == 5)
@@ -795,7 +803,7 @@ def main():
     # ---- CPU baseline (rank 0, N = 1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
-        cpu = cpu_baseline_sample()
+        cpu = cpu_baseline_sample(min(args.n_log2, 28))
 
     sweep_lines = []
     if args.sweep and world == 1:
