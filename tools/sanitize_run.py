@@ -25,4 +25,31 @@ with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=3, batch=3000)
     check(*gpu_roundtrip(t, keys, vals, q))
 with wd.Table(capacity_for(n, 0.9), 1, 8, batch=3000) as t:
     check(*gpu_roundtrip(t, keys, vals, q, host=True))
+# round 2 paths: V = 16 one-lane windows, the sliced insert with two chunks overlapped
+# (forced small chunks are env-only, so two calls), the |g| = 32 tail launch, the
+# copy-engine exchange, the _sharded calls, erase through the staged reverse path
+with wd.Table(capacity_for(n, 0.9), 1, 16) as t:
+    t.set_option(wd.WD_OPT_SLOTS_PER_LANE, 16)
+    check(*gpu_roundtrip(t, keys, vals, q))
+for tail in (1, 2):
+    with wd.Table(capacity_for(n, 0.99), 1, 4) as t:
+        t.set_option(wd.WD_OPT_TAIL, tail)
+        check(*gpu_roundtrip(t, keys, vals, q))
+with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=3, batch=3000, exchange=1) as t:
+    check(*gpu_roundtrip(t, keys, vals, q))
+    er = t.erase(torch.from_numpy(q[: n // 2].view(np.int32)).cuda())
+    torch.cuda.synchronize()
+    assert np.array_equal(er.cpu().numpy().astype(bool), cf[: n // 2].astype(bool))
+with wd.Table(capacity_for(n, 0.9), group_size=4, loopback_shards=2, batch=4000) as t:
+    import wdgen.gpu as gg
+    half = n // 2
+    ks = [gg.unique_keys(half, 1, start=r * half) for r in range(2)]
+    vs = [gg.values(half, 2, start=r * half) for r in range(2)]
+    t.insert_sharded(ks, vs)
+    vo = [torch.empty(half, dtype=torch.int32, device="cuda") for _ in range(2)]
+    fo = [torch.empty(half, dtype=torch.uint8, device="cuda") for _ in range(2)]
+    t.retrieve_sharded(ks, vo, fo)
+    torch.cuda.synchronize()
+    for r in range(2):
+        assert gg.check_unique(ks[r], vo[r], fo[r], n, 1, 2)[0] == 0
 print("sanitize run ok")
