@@ -220,8 +220,8 @@ typedef enum {
                                 inserted with one probe launch per slice (better L2 reuse); the
                                 probing of each key is unchanged.  0 (default): for tables > 512 MB
                                 and calls of >= 2^26 pairs (unless the span read-ahead
-                                applies), the power of two that makes a slice <= 160 MB
-                                (16 for config 2's 2.3 GB), at most 32, and off when a slice
+                                applies), the power of two that makes a slice <= 80 MB
+                                (32 for config 2's 2.3 GB), at most 32, and off when a slice
                                 would exceed 300 MB (measured slower);
                                 1: off; 2..32: that many slices.  Uses 8 B of scratch per pair,
                                 two buffers of at most 2^28 pairs (grouping of the next chunk

@@ -595,8 +595,9 @@ wd_status_t probe_soa(wd_table* t, Shard& s, int op, const wd::InSoA& in, uint32
 // read-ahead (|g| = 1), whose gain the sliced launches (InBucket) do not have.  The slice
 // count follows the table: slices of ~128-280 MB pay, slices of ~540 MB are SLOWER than no
 // slicing (profiles/r02/capacity_knee.md, 2^29 pairs at alpha 0.5 into 8.6 GB: 16 slices
-// 9.9, none 17.1, 32 slices 22.1 G inserts/s); at most 32 slices, so tables above ~9.6 GB
-// are not sliced.
+// 9.9, none 17.1, 32 slices 22.1 G inserts/s); slices of <= 80 MB where possible (2^28 pairs
+// into 2.3 GB: 8 / 16 / 32 slices -> 16.7 / 19.65 / 19.86 G/s — the probes gain more than
+// the 32-way multisplit loses); at most 32 slices, so tables above ~9.6 GB are not sliced.
 int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
   if (op != OP_INSERT || t->serial || t->slices == 1) return 1;
   if (t->slices > 1) return t->slices;
@@ -605,7 +606,7 @@ int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
   const int v = choose_v(t, s, t->G_used, true);
   if (choose_span(t, s, t->G_used, v) == 2) return 1;
   int nbk = 2;
-  while (nbk < wd::kMaxShards && tb / nbk > 160e6) nbk *= 2;
+  while (nbk < wd::kMaxShards && tb / nbk > 80e6) nbk *= 2;
   if (tb / nbk > 300e6) return 1;
   return nbk;
 }

@@ -496,7 +496,7 @@ def test_slice_grouped_insert_chunks(wd):
     n, ks, vs = (1 << 28) + 12_345, 71, 72            # two 2^28-pair chunks (ragged second)
     keys, vals = gg.unique_keys(n, ks), gg.values(n, vs)
     with wd.Table(capacity_for(n, 0.95), 1, 16) as t:
-        assert t.get_option(wd.WD_OPT_SLICES) == 0                 # auto -> 16 here (2.4 GB)
+        assert t.get_option(wd.WD_OPT_SLICES) == 0                 # auto -> 32 here (2.4 GB)
         t.insert(keys, vals)
         del vals
         q = gg.interleaved_queries(n, ks, start=n - (1 << 24), count=1 << 25)

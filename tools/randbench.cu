@@ -173,6 +173,45 @@ void run_chase2(unsigned long long* buf, uint64_t bytes, int grid, int kpc, uint
          grid * 256 / 148, keys / (ms * 1e-3) / 1e9, 2 * keys / (ms * 1e-3) / 1e9);
 }
 
+// atomics only: every lane issues D independent 64-bit CAS (succeeding: the expected value is
+// read first by the same lane... no — plain CAS on random slots, alternating values so each
+// succeeds or fails with ~1/2), or atomicAdd, on random 8-B slots of the buffer: the L2's
+// random atomic throughput, the floor of an insert's claim (one CAS per new key).
+template <int D, int OP>
+__global__ void __launch_bounds__(256) atom_only(unsigned long long* buf, uint64_t nslot, int iters,
+                                                 unsigned long long* sink) {
+  const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned long long acc = 0;
+  for (int it = 0; it < iters; ++it) {
+    unsigned long long r[D];
+#pragma unroll
+    for (int d = 0; d < D; ++d) {
+      const uint32_t h = hash32(tid * 2654435761u + (it * D + d) * 40503u + 17u);
+      unsigned long long* p = buf + ((uint64_t(h) * nslot) >> 32);
+      if (OP == 0) r[d] = atomicCAS(p, 0xFFFFFFFFFFFFFFFFull, uint64_t(tid));
+      else r[d] = atomicAdd(p, 1ull);
+    }
+#pragma unroll
+    for (int d = 0; d < D; ++d) acc += r[d];
+  }
+  if (acc == 42) sink[0] = acc;
+}
+template <int D, int OP>
+void run_atom(unsigned long long* buf, uint64_t bytes, int grid, int iters, unsigned long long* sink) {
+  const uint64_t nslot = bytes / 8;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a); cudaEventCreate(&b);
+  atom_only<D, OP><<<grid, 256>>>(buf, nslot, 2, sink);
+  cudaEventRecord(a);
+  atom_only<D, OP><<<grid, 256>>>(buf, nslot, iters, sink);
+  cudaEventRecord(b);
+  cudaEventSynchronize(b);
+  float ms; cudaEventElapsedTime(&ms, a, b);
+  const double ops = double(grid) * 256 * D * iters;
+  printf("%.4fGB %s-only D=%d (%d thr/SM): %6.1f G atomics/s\n", bytes / 1e9, OP == 0 ? "cas" : "add",
+         D, grid * 256 / 148, ops / (ms * 1e-3) / 1e9);
+}
+
 template <int D, int MODE, int WB, int AB>
 void run(const char* name, unsigned long long* buf, uint64_t bytes, int grid, int iters,
          unsigned long long* sink) {
@@ -206,6 +245,11 @@ int main(int argc, char** argv) {
     cudaMemset(buf, 0xff, bytes);
     const int grid = sms * 8;
     const int it = 32;
+    run_atom<4, 0>(buf, bytes, grid, it, sink);
+    run_atom<8, 0>(buf, bytes, grid, it, sink);
+    run_atom<8, 1>(buf, bytes, grid, it, sink);
+    run_atom<8, 0>(buf, bytes, sms * 4, it, sink);
+    if (getenv("RB_ATOM_ONLY")) { cudaFree(buf); continue; }
     run<8, 0, 8, 32>("read", buf, bytes, grid, it, sink);
     run<8, 0, 32, 32>("read", buf, bytes, grid, it, sink);
     run<8, 0, 32, 64>("read", buf, bytes, grid, it, sink);
