@@ -7,7 +7,7 @@ O=gpurun_out/$T
 mkdir -p $O
 timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
   -c 200 --csv --log-file $O/launches.csv python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu > $O/ncu_list.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:probe_ -s 17 -c 2 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:probe_ -s 31 -c 2 \
   -o $O/full python bench.py --steps 1 --warmup 1 --no-e2e --no-cpu > $O/ncu_full.log 2>&1
 ncu -i $O/full.ncu-rep --page raw --csv > $O/raw.csv 2>/dev/null
 ncu -i $O/full.ncu-rep --page details --csv > $O/details.csv 2>/dev/null
