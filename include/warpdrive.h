@@ -257,6 +257,14 @@ typedef enum {
                                 more than the shorter chains save (profiles/r02/
                                 tail_launch.md); T >= 1: that threshold.  Uses a 24 MB spill
                                 list per shard (keys beyond 2^20 spills just keep probing). */
+    WD_OPT_AUTO_REBUILD = 15, /* P:63 "the whole data structure is invalidated followed by a
+                                subsequent reconstruction with a distinct hash function":
+                                1 = after an insert call that left keys behind (Line 26) while
+                                live keys + those keys still fit the capacity (e.g. tombstones
+                                fill the probe sequences), rebuild with a new seed and re-insert
+                                them (up to 4 times).  Makes wd_insert synchronous.  0
+                                (default): off, the sticky WD_ERR_TABLE_FULL is reported.
+                                Single-process tables only (not rank mode). */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -278,6 +278,8 @@ void shard_free(Shard& s) {
   if (s.counters) cudaFree(s.counters);
   if (s.tail) cudaFree(s.tail);
   if (s.tail_count) cudaFree(s.tail_count);
+  if (s.fail_list) cudaFree(s.fail_list);
+  if (s.fail_count) cudaFree(s.fail_count);
   for (int i = 0; i < kStage; ++i) {
     if (s.ev_h2d[i]) cudaEventDestroy(s.ev_h2d[i]);
     if (s.ev_free[i]) cudaEventDestroy(s.ev_free[i]);
@@ -1266,6 +1268,110 @@ const char* op_name(int op) {
   return op == OP_INSERT ? "wd_insert" : op == OP_RETRIEVE ? "wd_retrieve" : "wd_erase";
 }
 
+wd_status_t do_op_plain(wd_table* t, int op, const IO& io, cudaStream_t stream) {
+  if (t->m == 1) {
+    if (io.n == 0) return WD_OK;
+    return single_op(t, op, io, stream);
+  }
+  std::vector<IO> ios;
+  split_io(t, io, ios);
+  return cascade_op(t, op, ios, stream);
+}
+
+extern "C" wd_status_t wd_rebuild(wd_table_t* t, uint32_t seed, wd_stream_t stream);
+
+// "In the unlikely case that the probing scheme cannot determine an empty slot for
+// n < c the whole data structure is invalidated followed by a subsequent reconstruction with
+// a distinct hash function."  With WD_OPT_AUTO_REBUILD an insert call that left keys behind
+// (Line 26) while the table still has room — e.g. tombstones of earlier deletions fill the
+// probe sequences (reading C9') — is followed, synchronously, by wd_rebuild with a new seed
+// (the tombstones go) and a re-insert of the keys recorded at Line 26.
+wd_status_t insert_auto_rebuild(wd_table* t, const IO& io, cudaStream_t stream) {
+  for (auto& s : t->local) {
+    DeviceGuard g(s.device);
+    if (!s.fail_list) {
+      CK(cudaMalloc(&s.fail_list, size_t(kFailCap) * sizeof(unsigned long long)));
+      CK(cudaMalloc(&s.fail_count, sizeof(unsigned long long)));
+    }
+    CK(cudaStreamSynchronize(stream));
+    CK(cudaMemset(s.fail_count, 0, sizeof(unsigned long long)));
+  }
+  TRY(do_op_plain(t, OP_INSERT, io, stream));
+  for (int attempt = 0; attempt < 4; ++attempt) {
+    // how many keys were left behind, and were they all recorded?
+    uint64_t failed = 0, live = 0;
+    bool recorded = true;
+    std::vector<unsigned long long> nfail(t->local.size(), 0);
+    for (size_t r = 0; r < t->local.size(); ++r) {
+      Shard& s = t->local[r];
+      DeviceGuard g(s.device);
+      CK(cudaStreamSynchronize(stream));
+      CK(cudaDeviceSynchronize());
+      unsigned long long c[wd::CNT_N], fc = 0;
+      CK(cudaMemcpy(c, s.counters, sizeof c, cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(&fc, s.fail_count, sizeof fc, cudaMemcpyDeviceToHost));
+      failed += c[wd::CNT_FAIL];
+      live += c[wd::CNT_NEW] - c[wd::CNT_ERASED];
+      nfail[r] = fc;
+      recorded = recorded && fc == c[wd::CNT_FAIL] && fc <= kFailCap;
+    }
+    if (failed == 0) return WD_OK;
+    if (!recorded || live + failed > wd_capacity(t))   // truly full: keep the sticky error
+      return fail(WD_ERR_TABLE_FULL, "%llu inserts exhausted p_max with %llu of %llu slots live",
+                  (unsigned long long)failed, (unsigned long long)live,
+                  (unsigned long long)wd_capacity(t));
+    // set the recorded pairs aside, rebuild with a distinct hash, re-insert them
+    std::vector<unsigned long long*> keep(t->local.size(), nullptr), kcnt(t->local.size(), nullptr);
+    auto release = [&]() {
+      for (size_t r = 0; r < t->local.size(); ++r) {
+        DeviceGuard g(t->local[r].device);
+        if (keep[r]) cudaFree(keep[r]);
+        if (kcnt[r]) cudaFree(kcnt[r]);
+      }
+    };
+    for (size_t r = 0; r < t->local.size(); ++r) {
+      Shard& s = t->local[r];
+      DeviceGuard g(s.device);
+      cudaError_t e = cudaMalloc(&keep[r], std::max<uint64_t>(nfail[r], 1) * 8);
+      if (e == cudaSuccess) e = cudaMalloc(&kcnt[r], 8);
+      if (e == cudaSuccess && nfail[r])
+        e = cudaMemcpy(keep[r], s.fail_list, nfail[r] * 8, cudaMemcpyDeviceToDevice);
+      if (e == cudaSuccess) e = cudaMemcpy(kcnt[r], &nfail[r], 8, cudaMemcpyHostToDevice);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        release();
+        return fail(WD_ERR_OUT_OF_MEMORY, "auto rebuild: %s", cudaGetErrorString(e));
+      }
+    }
+    // the failure record restarts: failures of the rebuild's own re-insert and of the
+    // re-insert below are recorded again and handled by the next attempt
+    wd_status_t st = WD_OK;
+    for (size_t r = 0; st == WD_OK && r < t->local.size(); ++r) {
+      Shard& s = t->local[r];
+      DeviceGuard g(s.device);
+      if (cudaMemset(s.counters + wd::CNT_FAIL, 0, 8) != cudaSuccess ||
+          cudaMemset(s.fail_count, 0, 8) != cudaSuccess)
+        st = fail(WD_ERR_CUDA, "auto rebuild: counter reset");
+    }
+    ++t->rebuilds;
+    const uint32_t seed = t->local[0].hseed + 0x9E3779B9u * t->rebuilds;
+    if (st == WD_OK) st = wd_rebuild(t, seed, reinterpret_cast<wd_stream_t>(stream));
+    for (size_t r = 0; st == WD_OK && r < t->local.size(); ++r) {
+      Shard& s = t->local[r];
+      DeviceGuard g(s.device);
+      if (nfail[r]) {
+        const wd::InSeg<true> in{keep[r], kcnt[r], nfail[r], 1};
+        st = launch_probe<true>(t, s, in, wd::OutNone{}, nfail[r], s.s_main);
+      }
+      if (st == WD_OK && cudaStreamSynchronize(s.s_main) != cudaSuccess)
+        st = fail(WD_ERR_CUDA, "auto rebuild: re-insert");
+    }
+    release();
+    TRY(st);
+  }
+  return fail(WD_ERR_TABLE_FULL, "auto rebuild: inserts still fail after 4 reconstructions");
+}
+
 wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* vals,
                   uint32_t* vout, uint8_t* fout, uint64_t n, cudaStream_t stream) {
   if (!t) return fail(WD_ERR_INVALID_ARG, "null table");
@@ -1274,13 +1380,8 @@ wd_status_t do_op(wd_table* t, int op, const uint32_t* keys, const uint32_t* val
   io.keys = keys; io.vals = vals; io.vout = vout; io.fout = fout; io.n = n;
   TRY(classify_io(t, op == OP_INSERT, io, -1));
   pick_group_size(t, op, n);
-  if (t->m == 1) {
-    if (n == 0) return WD_OK;
-    return single_op(t, op, io, stream);
-  }
-  std::vector<IO> ios;
-  split_io(t, io, ios);
-  return cascade_op(t, op, ios, stream);
+  if (op == OP_INSERT && t->auto_rebuild && n) return insert_auto_rebuild(t, io, stream);
+  return do_op_plain(t, op, io, stream);
 }
 
 // The paper's device-sided cascades: every local shard brings its own
@@ -1771,6 +1872,11 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       if (v < 0 || v > 1000) return fail(WD_ERR_INVALID_ARG, "tail %lld", (long long)v);
       t->tail = int(v);
       return WD_OK;
+    case WD_OPT_AUTO_REBUILD:
+      if (v && t->mode == MODE_RANK)
+        return fail(WD_ERR_UNSUPPORTED, "automatic rebuild is single-process only");
+      t->auto_rebuild = v != 0;
+      return WD_OK;
     case WD_OPT_EXCHANGE:
       if (v < 0 || v > 2) return fail(WD_ERR_INVALID_ARG, "exchange %lld", (long long)v);
       if (v == 2 && t->mode == MODE_LOOPBACK)
@@ -1804,6 +1910,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_EXCHANGE: return t->exchange;
     case WD_OPT_PHASE_TIMING: return t->phase_on ? 1 : 0;
     case WD_OPT_TAIL: return t->tail;
+    case WD_OPT_AUTO_REBUILD: return t->auto_rebuild ? 1 : 0;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;
     case WD_OPT_LOCAL_SHARDS: return int64_t(t->local.size());

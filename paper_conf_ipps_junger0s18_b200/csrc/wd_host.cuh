@@ -125,6 +125,8 @@ struct Shard {
   cudaEvent_t ev_ready[2] = {}, ev_pdone[2] = {}, ev_done[2] = {}, ev_unperm[2] = {};
   bool pdone_rec[2] = {}, unperm_rec[2] = {};
   wd::TailEntry* tail = nullptr;   // spill list of long probe chains (WD_OPT_TAIL)
+  unsigned long long* fail_list = nullptr;    // inserts that hit Line 26 (WD_OPT_AUTO_REBUILD)
+  unsigned long long* fail_count = nullptr;
   unsigned long long* tail_count = nullptr;
   void* comm_fwd = nullptr;        // ncclComm_t of the forward / reverse transpositions
   void* comm_rev = nullptr;
@@ -176,6 +178,8 @@ struct wd_table {
   // exact counts after an all-gather of T; the north star's NCCL path)
   int exchange = 0;
   int tail = 0;             // WD_OPT_TAIL: regions before a chain is spilled (0: off)
+  bool auto_rebuild = false;  // WD_OPT_AUTO_REBUILD
+  uint32_t rebuilds = 0;      // automatic rebuilds so far (new seeds are derived from it)
   uint32_t tail_now = 0;    // spill threshold of the launch being issued (launch_probe)
   // per-phase CUDA-event timing (WD_OPT_PHASE_TIMING, wd_phase_times): begin/end event pairs
   // recorded on the stream each phase runs on; events are pooled per device
@@ -229,6 +233,7 @@ int blocks_per_sm(K kern, size_t dyn_smem = 0) {
 
 // ------------------------------------------------------------------ probe dispatch
 constexpr uint32_t kTailCap = 1u << 20;   // spill-list entries per shard (24 MB)
+constexpr uint32_t kFailCap = 1u << 20;   // failed-insert list per shard (8 MB, auto rebuild)
 
 template <int G, int V, int K, bool INSERT, class In, class Out, int S = 1>
 wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
@@ -239,7 +244,8 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
   // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
   wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags, s.hseed, t->align,
-                   t->tail_now, kTailCap, s.tail, s.tail_count};
+                   t->tail_now, kTailCap, s.tail, s.tail_count,
+                   INSERT && t->auto_rebuild ? s.fail_list : nullptr, s.fail_count, kFailCap};
   int grid = 1, block = 32;
   if (!t->serial) {
     block = wd::kBlock;

@@ -126,3 +126,42 @@ def test_erase_loopback_and_host(wd, m):
     want = np.ones(n, np.uint8); want[::4] = 0
     assert np.array_equal(gf, want) and np.array_equal(gf2, want)
     assert np.array_equal(gv[want == 1], vals[want == 1]) and np.array_equal(gv2, gv)
+
+
+@pytest.mark.parametrize("G,shards", [(4, 1), (16, 1), (8, 3)])
+def test_auto_rebuild_on_table_full(wd, G, shards):
+    # an insert that cannot find an empty slot while n < c triggers a reconstruction
+    # with a distinct hash.  Tombstones (reading C9': not reused before a rebuild) fill the
+    # table: without WD_OPT_AUTO_REBUILD the later insert fails (sticky TABLE_FULL), with it
+    # the table rebuilds, re-inserts the keys left behind and ends exact.
+    n = 60_000
+    keys, vals = wdgen.unique_keys(n, 201), wdgen.values(n, 202)
+    more = wdgen.unique_keys(n // 2, 201, start=n)
+    mvals = wdgen.values(n // 2, 203)
+    cap = capacity_for(n, 0.97)
+    kw = {"loopback_shards": shards} if shards > 1 else {}
+    results = {}
+    for auto in (0, 1):
+        with wd.Table(cap, group_size=G, **kw) if shards > 1 else wd.Table(cap, 1, G) as t:
+            if shards > 1:
+                t.set_option(wd.WD_OPT_BATCH, 10_000)
+            t.set_option(wd.WD_OPT_AUTO_REBUILD, auto)
+            assert t.get_option(wd.WD_OPT_AUTO_REBUILD) == auto
+            t.insert(to_dev(keys), to_dev(vals))
+            _erase(t, keys[: n // 2])                      # half the table becomes tombstones
+            assert t.sync() == 0 and t.size() == n - n // 2
+            if auto:
+                t.insert(to_dev(more), to_dev(mvals))      # recovers: no error
+            else:
+                t.insert(to_dev(more), to_dev(mvals))
+            st = t.sync()
+            results[auto] = st
+            if auto:
+                assert st == 0, wd._lib.wd_last_error_message()
+                assert t.size() == n
+                q = np.concatenate([keys, more])
+                gv, gf = gpu_roundtrip(t, np.zeros(0, np.uint32), np.zeros(0, np.uint32), q)
+                want = np.concatenate([np.zeros(n // 2, np.uint8), np.ones(n - n // 2 + n // 2, np.uint8)])
+                assert np.array_equal(gf, want)
+                assert np.array_equal(gv[n // 2: n], vals[n // 2:]) and np.array_equal(gv[n:], mvals)
+    assert results[0] == wd.WD_ERR_TABLE_FULL
