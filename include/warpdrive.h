@@ -219,10 +219,11 @@ typedef enum {
                                 is grouped by table slice of the keys' first region (Line 5) and
                                 inserted with one probe launch per slice (better L2 reuse); the
                                 probing of each key is unchanged.  0 (default): for tables > 512 MB
-                                and calls of >= 2^26 pairs (unless the span read-ahead
-                                applies), the power of two that makes a slice <= 80 MB
-                                (32 for config 2's 2.3 GB), at most 32, and off when a slice
-                                would exceed 300 MB (measured slower);
+                                (> 1 GB where the span read-ahead applies) and calls of
+                                >= 2^26 pairs, the power of two that makes a slice <= 80 MB
+                                for |g| = 16 on line-aligned tables (32 for config 2's
+                                2.3 GB) or <= 160 MB otherwise, at most 32, and off when a
+                                slice would exceed 300 MB (measured slower);
                                 1: off; 2..32: that many slices.  Uses 8 B of scratch per pair,
                                 two buffers of at most 2^28 pairs (grouping of the next chunk
                                 overlaps the probing of this one), kept for the table's lifetime
@@ -248,15 +249,8 @@ typedef enum {
                                 Results are identical in all three modes. */
     WD_OPT_PHASE_TIMING = 13, /* 1: record CUDA events around every phase of every call (see
                                 wd_phase_times); 0 (default): off */
-    WD_OPT_TAIL = 14,        /* long probe chains (the probing scheme does not depend on
-                                |g|): a key still probing when it enters region number T is
-                                handed to a second launch that probes with |g| = 32, one window
-                                per region (same regions, same order, same leftmost decisions);
-                                a call ends with its longest chain, so small calls get faster.
-                                0 (default): off — measured on B200, the extra launch costs
-                                more than the shorter chains save (profiles/r02/
-                                tail_launch.md); T >= 1: that threshold.  Uses a 24 MB spill
-                                list per shard (keys beyond 2^20 spills just keep probing). */
+    /* 14: reserved (a |g| = 32 launch for long probe chains was measured slower and removed,
+       profiles/r02/tail_launch.md) */
     WD_OPT_AUTO_REBUILD = 15, /* P:63 "the whole data structure is invalidated followed by a
                                 subsequent reconstruction with a distinct hash function":
                                 1 = after an insert call that left keys behind (Line 26) while

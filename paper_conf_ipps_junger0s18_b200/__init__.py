@@ -33,7 +33,6 @@ WD_OPT_KEYS_IN_FLIGHT, WD_OPT_PART_SEED, WD_OPT_PART_MODE, WD_OPT_PROBE_MODE = 4
 WD_OPT_KERNEL_FLAGS, WD_OPT_SLOTS_PER_LANE, WD_OPT_SPAN, WD_OPT_SLICES = 8, 9, 10, 11
 WD_OPT_EXCHANGE = 12
 WD_OPT_PHASE_TIMING = 13
-WD_OPT_TAIL = 14
 WD_OPT_AUTO_REBUILD = 15
 PHASES = ["h2d", "group", "multisplit", "exchange", "probe", "reverse", "unpermute", "d2h",
           "probe_query"]

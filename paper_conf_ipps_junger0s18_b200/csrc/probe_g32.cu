@@ -5,5 +5,4 @@
 
 namespace wdi {
 WD_PROBE_COMBOS(WD_PROBE_INST, 32)
-WD_TAIL_COMBOS(WD_PROBE_INST)
 }  // namespace wdi

@@ -169,17 +169,6 @@ void l2_fetch_release(int device) {
   h.set = false;
 }
 
-// ------------------------------------------------------------------ long-chain spill list
-wd_status_t tail_prepare(wd_table* t, Shard& s, cudaStream_t st) {
-  (void)t;
-  if (!s.tail) {
-    CK(cudaMalloc(&s.tail, size_t(kTailCap) * sizeof(wd::TailEntry)));
-    CK(cudaMalloc(&s.tail_count, sizeof(unsigned long long)));
-  }
-  CK(cudaMemsetAsync(s.tail_count, 0, sizeof(unsigned long long), st));
-  return WD_OK;
-}
-
 // ------------------------------------------------------------------ shard lifetime
 wd_status_t shard_init(wd_table* t, Shard& s, int id, int device, uint64_t cap,
                        cudaStream_t shared_main) {
@@ -276,8 +265,6 @@ void shard_free(Shard& s) {
   }
   if (s.slots) cudaFree(s.slots);
   if (s.counters) cudaFree(s.counters);
-  if (s.tail) cudaFree(s.tail);
-  if (s.tail_count) cudaFree(s.tail_count);
   if (s.fail_list) cudaFree(s.fail_list);
   if (s.fail_count) cudaFree(s.fail_count);
   for (int i = 0; i < kStage; ++i) {
@@ -605,10 +592,16 @@ int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
   if (t->slices > 1) return t->slices;
   const double tb = double(s.cap) * sizeof(unsigned long long);
   if (tb <= double(512ull << 20) || n < (1ull << 26)) return 1;
+  // the plain launch's span read-ahead (|g| = 1) wins up to ~1 GB, slicing beyond it
+  // (|g| = 1, alpha 0.95: 2^26 pairs 7.5 vs 7.45, 2^27 5.7 vs 7.5, 2^28 5.2 vs 7.5 G/s)
   const int v = choose_v(t, s, t->G_used, true);
-  if (choose_span(t, s, t->G_used, v) == 2) return 1;
+  if (choose_span(t, s, t->G_used, v) == 2 && tb <= 1.0e9) return 1;
+  // <= 80 MB slices where the launches read one line per lane (|g| = 16 on a line-aligned
+  // table: 16 -> 32 slices 19.65 -> 19.86 G/s at alpha 0.95, 12.5 -> 13.3 at 0.99); <= 160 MB
+  // otherwise (|g| = 4: 16 slices 15.5, 32 slices 13.4 G/s)
+  const double target = (t->G_used == 16 && t->align == 16) ? 80e6 : 160e6;
   int nbk = 2;
-  while (nbk < wd::kMaxShards && tb / nbk > 80e6) nbk *= 2;
+  while (nbk < wd::kMaxShards && tb / nbk > target) nbk *= 2;
   if (tb / nbk > 300e6) return 1;
   return nbk;
 }
@@ -1868,10 +1861,6 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
     case WD_OPT_PHASE_TIMING:
       t->phase_on = v != 0;
       return WD_OK;
-    case WD_OPT_TAIL:
-      if (v < 0 || v > 1000) return fail(WD_ERR_INVALID_ARG, "tail %lld", (long long)v);
-      t->tail = int(v);
-      return WD_OK;
     case WD_OPT_AUTO_REBUILD:
       if (v && t->mode == MODE_RANK)
         return fail(WD_ERR_UNSUPPORTED, "automatic rebuild is single-process only");
@@ -1909,7 +1898,6 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_SLICES: return t->slices;
     case WD_OPT_EXCHANGE: return t->exchange;
     case WD_OPT_PHASE_TIMING: return t->phase_on ? 1 : 0;
-    case WD_OPT_TAIL: return t->tail;
     case WD_OPT_AUTO_REBUILD: return t->auto_rebuild ? 1 : 0;
     case WD_OPT_N_SHARDS: return t->m;
     case WD_OPT_RANK: return t->rank;

@@ -124,10 +124,8 @@ struct Shard {
   cudaEvent_t ev_row = nullptr, ev_col = nullptr;
   cudaEvent_t ev_ready[2] = {}, ev_pdone[2] = {}, ev_done[2] = {}, ev_unperm[2] = {};
   bool pdone_rec[2] = {}, unperm_rec[2] = {};
-  wd::TailEntry* tail = nullptr;   // spill list of long probe chains (WD_OPT_TAIL)
   unsigned long long* fail_list = nullptr;    // inserts that hit Line 26 (WD_OPT_AUTO_REBUILD)
   unsigned long long* fail_count = nullptr;
-  unsigned long long* tail_count = nullptr;
   void* comm_fwd = nullptr;        // ncclComm_t of the forward / reverse transpositions
   void* comm_rev = nullptr;
   bool l2_held = false;            // holds the device's L2 fetch-granularity setting
@@ -177,10 +175,8 @@ struct wd_table {
   // "asynchronous inter-GPU copies"), 2 staged buffers + NCCL send/recv (all-to-all(v) of
   // exact counts after an all-gather of T; the north star's NCCL path)
   int exchange = 0;
-  int tail = 0;             // WD_OPT_TAIL: regions before a chain is spilled (0: off)
   bool auto_rebuild = false;  // WD_OPT_AUTO_REBUILD
   uint32_t rebuilds = 0;      // automatic rebuilds so far (new seeds are derived from it)
-  uint32_t tail_now = 0;    // spill threshold of the launch being issued (launch_probe)
   // per-phase CUDA-event timing (WD_OPT_PHASE_TIMING, wd_phase_times): begin/end event pairs
   // recorded on the stream each phase runs on; events are pooled per device
   bool phase_on = false;
@@ -232,7 +228,6 @@ int blocks_per_sm(K kern, size_t dyn_smem = 0) {
 }
 
 // ------------------------------------------------------------------ probe dispatch
-constexpr uint32_t kTailCap = 1u << 20;   // spill-list entries per shard (24 MB)
 constexpr uint32_t kFailCap = 1u << 20;   // failed-insert list per shard (8 MB, auto rebuild)
 
 template <int G, int V, int K, bool INSERT, class In, class Out, int S = 1>
@@ -244,7 +239,6 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
   // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
   wd::TableView tv{s.slots, static_cast<uint32_t>(s.nb), pmax, t->kflags, s.hseed, t->align,
-                   t->tail_now, kTailCap, s.tail, s.tail_count,
                    INSERT && t->auto_rebuild ? s.fail_list : nullptr, s.fail_count, kFailCap};
   int grid = 1, block = 32;
   if (!t->serial) {
@@ -380,18 +374,6 @@ wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, 
   launch_probe_g<G, I, IN, OUT>(wd_table*, Shard&, const IN&, const OUT&, uint64_t, cudaStream_t)
 #define WD_PROBE_EXTERN(G, I, IN, OUT) extern template wd_status_t WD_PROBE_SIG(G, I, IN, OUT);
 #define WD_PROBE_INST(G, I, IN, OUT) template wd_status_t WD_PROBE_SIG(G, I, IN, OUT);
-// the wide launch of spilled long chains (|g| = 32), for every output type
-#define WD_TAIL_COMBOS(X)                                     \
-  X(32, true, wd::InTail, wd::OutNone)                        \
-  X(32, false, wd::InTail, wd::OutSoA)                        \
-  X(32, false, wd::InTail, wd::OutErase<wd::OutSoA>)          \
-  X(32, false, wd::InTail, wd::OutPacked)                     \
-  X(32, false, wd::InTail, wd::OutErase<wd::OutPacked>)       \
-  X(32, false, wd::InTail, wd::OutLocalPacked)                \
-  X(32, false, wd::InTail, wd::OutErase<wd::OutLocalPacked>)
-#ifndef WD_PROBE_TU
-WD_TAIL_COMBOS(WD_PROBE_EXTERN)
-#endif
 #ifndef WD_PROBE_TU
 WD_PROBE_COMBOS(WD_PROBE_EXTERN, 1)
 WD_PROBE_COMBOS(WD_PROBE_EXTERN, 2)
@@ -401,37 +383,9 @@ WD_PROBE_COMBOS(WD_PROBE_EXTERN, 16)
 WD_PROBE_COMBOS(WD_PROBE_EXTERN, 32)
 #endif
 
-// Spill threshold for this table (WD_OPT_TAIL): off by default — measured on B200
-// (tools/gpu_tail.sh, profiles/r02/tail_launch.md) the extra launch costs more than the
-// shortened chains save, even for L2-resident config-1 calls.
-inline uint32_t tail_after(const wd_table* t, const Shard& s) {
-  if (t->serial || t->G_used >= 32) return 0;
-  return t->tail > 0 ? uint32_t(t->tail) : 0u;
-}
-wd_status_t tail_prepare(wd_table* t, Shard& s, cudaStream_t st);   // warpdrive.cu
-
-template <bool INSERT, class In, class Out>
-wd_status_t launch_probe_main(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
-                              cudaStream_t st);
-
 template <bool INSERT, class In, class Out>
 wd_status_t launch_probe(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                          cudaStream_t st) {
-  const uint32_t ta = tail_after(t, s);
-  if (ta == 0) return launch_probe_main<INSERT>(t, s, in, out, n_hint, st);
-  TRY(tail_prepare(t, s, st));                  // spill counter = 0 (stream-ordered)
-  t->tail_now = ta;
-  const wd_status_t r = launch_probe_main<INSERT>(t, s, in, out, n_hint, st);
-  t->tail_now = 0;
-  TRY(r);
-  // the wide launch: |g| = 32, one window per region, resuming every spilled chain
-  return launch_probe_g<32, INSERT>(t, s, wd::InTail{s.tail, s.tail_count, kTailCap}, out,
-                                    std::min<uint64_t>(n_hint, kTailCap), st);
-}
-
-template <bool INSERT, class In, class Out>
-wd_status_t launch_probe_main(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
-                              cudaStream_t st) {
   switch (t->G_used) {
     case 1: return launch_probe_g<1, INSERT>(t, s, in, out, n_hint, st);
     case 2: return launch_probe_g<2, INSERT>(t, s, in, out, n_hint, st);

@@ -193,17 +193,55 @@ def test_loopback_rejects_nccl_exchange(wd):
             t.set_option(wd.WD_OPT_EXCHANGE, 3)
 
 
-@pytest.mark.parametrize("exchange", [0, 1])
-def test_loopback_tail_launch(wd, exchange):
-    # the wide tail launch inside the cascade: its answers go through the same reverse
-    # transposition (OutPacked / OutLocalPacked) as the main launch's
-    n = 120_007
-    keys, vals = wdgen.unique_keys(n, 141), wdgen.values(n, 142)
-    q = wdgen.interleaved_queries(n, 141)
-    with wd.Table(capacity_for(n, 0.99), group_size=4, loopback_shards=3, exchange=exchange) as t:
-        t.set_option(wd.WD_OPT_TAIL, 1)
-        t.set_option(wd.WD_OPT_BATCH, 30_000)
-        gv, gf = gpu_roundtrip(t, keys, vals, q)
+def test_phase_times_decomposition(wd):
+    # wd_phase_times (Fig. 11 decomposition): the phases each path runs are reported, with
+    # positive times; off by default; reading resets
+    import torch
+    import wdgen.gpu as gg
+    n = 1 << 22
+    keys, vals = gg.unique_keys(n, 301), gg.values(n, 302)
+    with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=2, batch=1 << 20,
+                  exchange=1) as t:
+        t.insert(keys, vals)
+        assert all(c == 0 for _, c in t.phase_times().values())      # off: nothing recorded
+        t.set_option(wd.WD_OPT_PHASE_TIMING, 1)
+        t.insert(keys, vals)
+        ph = t.phase_times()
+        assert {k for k, (ms, c) in ph.items() if c} == {"multisplit", "exchange", "probe"}
+        assert all(ms > 0 for ms, c in ph.values() if c)
+        vo = torch.empty(n, dtype=torch.int32, device="cuda")
+        fo = torch.empty(n, dtype=torch.uint8, device="cuda")
+        t.retrieve(keys, vo, fo)
+        ph = t.phase_times()
+        assert {k for k, (ms, c) in ph.items() if c} == {"multisplit", "exchange", "probe_query",
+                                                          "reverse", "unpermute"}
+        assert gg.check_unique(keys, vo, fo, n, 301, 302)[0] == 0
+    with wd.Table(capacity_for(n, 0.9), 1, 16) as t:
+        t.set_option(wd.WD_OPT_PHASE_TIMING, 1)
+        t.set_option(wd.WD_OPT_SLICES, 4)
+        t.insert(keys, vals)
+        assert {k for k, (ms, c) in t.phase_times().items() if c} == {"group", "probe"}
+        hk = keys.cpu().pin_memory()
+        t.retrieve(hk)
+        assert {k for k, (ms, c) in t.phase_times().items() if c} == {"h2d", "probe_query", "d2h"}
+
+
+def test_sharded_host_portions(wd):
+    # _sharded calls with pinned host portions: streamed per shard (a11) through the cascade
+    import torch
+    n_local, m = 70_001, 3
+    n = n_local * m
+    with wd.Table(capacity_for(n, 0.9), group_size=4, loopback_shards=m, batch=20_000) as t:
+        ks = [torch.from_numpy(wdgen.unique_keys(n_local, 311, start=r * n_local).view(np.int32)).pin_memory()
+              for r in range(m)]
+        vs = [torch.from_numpy(wdgen.values(n_local, 312, start=r * n_local).view(np.int32)).pin_memory()
+              for r in range(m)]
+        t.insert_sharded(ks, vs)
+        vo = [torch.empty(n_local, dtype=torch.int32).pin_memory() for _ in range(m)]
+        fo = [torch.empty(n_local, dtype=torch.uint8).pin_memory() for _ in range(m)]
+        t.retrieve_sharded(ks, vo, fo)
+        torch.cuda.synchronize()
         assert t.sync() == 0 and t.size() == n
-    cv, cf = oracle.expected_unique(q, n, 141, 142)
-    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+    for r in range(m):
+        cv, cf = oracle.expected_unique(ks[r].numpy().view(np.uint32), n, 311, 312)
+        assert np.array_equal(fo[r].numpy(), cf) and np.array_equal(vo[r].numpy().view(np.uint32), cv)

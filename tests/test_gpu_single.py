@@ -511,44 +511,3 @@ def test_slice_grouped_insert_chunks(wd):
         assert t.launches >= 2 * (3 + 16)                             # two sliced chunks
     cv, cf = oracle.expected_unique(qs, n, ks, vs)
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
-
-
-@pytest.mark.parametrize("G", [1, 2, 4, 8, 16])
-@pytest.mark.parametrize("tail", [1, 3, 0])
-def test_long_chain_tail_launch(wd, G, tail):
-    # WD_OPT_TAIL: keys still probing at region T are resumed by a |g| = 32 launch (one
-    # window per region).  The map must be exact for inserts (with duplicates and
-    # updates), hit and miss queries and erase, at alpha 0.99 where chains are long.
-    n = 150_001
-    keys, vals = wdgen.unique_keys(n, 131), wdgen.values(n, 132)
-    q = wdgen.interleaved_queries(n, 131)
-    with wd.Table(capacity_for(n, 0.99), 1, G) as t:
-        t.set_option(wd.WD_OPT_TAIL, tail)
-        assert t.get_option(wd.WD_OPT_TAIL) == tail
-        gv, gf = gpu_roundtrip(t, keys, vals, q)
-        assert t.sync() == 0 and t.size() == n
-        k2 = keys[::7].copy()                                    # updates of present keys
-        v2 = wdgen.values(k2.size, 133)
-        t.insert(to_dev(k2), to_dev(v2))
-        ov, of = t.retrieve(to_dev(k2))
-        assert np.array_equal(from_dev(ov), v2) and bool((of == 1).all())
-        t.insert(to_dev(keys[::7]), to_dev(vals[::7]))           # back to the originals
-        df = t.erase(to_dev(q[: n // 2]))
-        assert t.sync() == 0
-        assert t.size() == n - int(oracle.expected_unique(q[: n // 2], n, 131, 132)[1].sum())
-    cv, cf = oracle.expected_unique(q, n, 131, 132)
-    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
-    assert np.array_equal(df.cpu().numpy().astype(bool), cf[: n // 2].astype(bool))
-    # duplicates: v in V(k), size = #distinct
-    dk = wdgen.uniform_keys(200_000, 134) % np.uint32(90_000)
-    dv = wdgen.values(200_000, 135)
-    with wd.Table(capacity_for(np.unique(dk).size, 0.99), 1, G) as t:
-        t.set_option(wd.WD_OPT_TAIL, tail)
-        qq = np.arange(91_000, dtype=np.uint32)
-        gv, gf = gpu_roundtrip(t, dk, dv, qq)
-        m = oracle.Map(200_000, dup_mode=True)
-        m.insert(dk, dv)
-        assert t.sync() == 0 and t.size() == m.size()
-    ev, ef = m.retrieve(qq)
-    assert np.array_equal(gf, ef)
-    assert np.all(m.pair_status(qq[gf == 1], gv[gf == 1]) >= 1)

@@ -19,7 +19,7 @@ import paper_conf_ipps_junger0s18_b200 as wd  # noqa: E402
 import wdgen.gpu as gg  # noqa: E402
 
 OPT = {"slices": wd.WD_OPT_SLICES, "v": wd.WD_OPT_SLOTS_PER_LANE, "k": wd.WD_OPT_KEYS_IN_FLIGHT,
-       "span": wd.WD_OPT_SPAN, "mode": wd.WD_OPT_PROBE_MODE, "tail": wd.WD_OPT_TAIL,
+       "span": wd.WD_OPT_SPAN, "mode": wd.WD_OPT_PROBE_MODE,
        "flags": wd.WD_OPT_KERNEL_FLAGS}
 
 

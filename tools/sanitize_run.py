@@ -26,15 +26,11 @@ with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=3, batch=3000)
 with wd.Table(capacity_for(n, 0.9), 1, 8, batch=3000) as t:
     check(*gpu_roundtrip(t, keys, vals, q, host=True))
 # round 2 paths: V = 16 one-lane windows, the sliced insert with two chunks overlapped
-# (forced small chunks are env-only, so two calls), the |g| = 32 tail launch, the
+# (forced small chunks are env-only, so two calls), the
 # copy-engine exchange, the _sharded calls, erase through the staged reverse path
 with wd.Table(capacity_for(n, 0.9), 1, 16) as t:
     t.set_option(wd.WD_OPT_SLOTS_PER_LANE, 16)
     check(*gpu_roundtrip(t, keys, vals, q))
-for tail in (1, 2):
-    with wd.Table(capacity_for(n, 0.99), 1, 4) as t:
-        t.set_option(wd.WD_OPT_TAIL, tail)
-        check(*gpu_roundtrip(t, keys, vals, q))
 with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=3, batch=3000, exchange=1) as t:
     check(*gpu_roundtrip(t, keys, vals, q))
     er = t.erase(torch.from_numpy(q[: n // 2].view(np.int32)).cuda())
