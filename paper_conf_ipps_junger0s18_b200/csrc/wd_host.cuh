@@ -342,9 +342,13 @@ wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, 
                            cudaStream_t st) {
   // sliced bulk inserts (InBucket) on line-aligned tables: one lane reads the whole 128-B
   // window (V = 16, K = 1; tools/gpu_vk_sweep.sh: 2^28 pairs 18.8 -> 19.7 G inserts/s, 2^24
-  // 20.5 -> 22.8).  Not for queries from HBM: one lane per 128-B line drops them to 9 G/s.
+  // 20.5 -> 22.8) while the projected load stays <= 0.975 — above it, with longer chains, two
+  // lanes of 64 B and two keys in flight win (alpha 0.97 / 0.98 / 0.99: 17.7 / 15.9 / 13.4
+  // vs 17.1 / 16.2 / 14.9 G/s).  Not for queries from HBM: one lane per 128-B line drops them
+  // to 9 G/s.
   if constexpr (G == 16 && INSERT && std::is_same_v<In, wd::InBucket>)
-    if (t->spl == 0 && t->kif == 0 && t->probe_mode == 0 && t->align == 16)
+    if (t->spl == 0 && t->kif == 0 && t->probe_mode == 0 && t->align == 16 &&
+        double(t->est_size) <= 0.975 * double(s.cap))
       return launch_gv<G, 16, INSERT>(t, s, in, out, n_hint, st, 1);
   const int v = choose_v(t, s, G, INSERT), k = choose_k(t, s, G, v, INSERT);
   if constexpr (G >= 16)
