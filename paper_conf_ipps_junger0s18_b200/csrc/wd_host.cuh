@@ -326,8 +326,12 @@ inline int choose_v(const wd_table* t, const Shard& s, int G, bool insert) {
 inline int choose_k(const wd_table* t, const Shard& s, int G, int V, bool insert) {
   if (t->kif) return t->kif;
   const bool small = s.cap * sizeof(unsigned long long) <= (64ull << 20);
-  if (V == 1) return G <= 4 ? 8 : 4;
-  if (V == 2) return small ? 4 : (G <= 2 ? 8 : 4);
+  // |g| = 1 inserts into tables > 1 GB run slice-grouped (no span read-ahead): K = 4
+  // (2^28, alpha 0.95: 7.5 -> 9.7 G/s); queries and smaller tables keep K = 8 with the span.
+  if (V == 1) return (G == 1 && insert && double(s.cap) * 8 > 1.0e9) ? 4 : (G <= 4 ? 8 : 4);
+  // V = 2: K = 4 everywhere (K = 8 spills: |g| = 2 from HBM 10.1 -> 14.3 G inserts/s and
+  // 7.0 -> 10.4 G queries/s, tools/rates.py, profiles/r02/small_g.jsonl)
+  if (V == 2) return 4;
   // V = 4: K = 2 (4 blocks/SM for inserts).  Judged on the whole step (tools/ab_retrieve.py,
   // |g| = 8, 2^28): insert/retrieve K = 2/2 -> 13.7 / 22.6 G/s (17.1 G ops/s combined),
   // 4/4 -> 12.9 / 23.5 (16.7), 2/4 -> 13.7 / 21.9 (16.8).
