@@ -319,8 +319,10 @@ inline int choose_v(const wd_table* t, const Shard& s, int G, bool insert) {
     else if (t->probe_mode == 2 || small) v = G;
     else v = G >= 2 ? std::max(1, std::min(G / 2, insert && t->align < 16 ? 4 : 8)) : 1;
     if (G == 2 && t->probe_mode == 0) v = 2;
+    // |g| = 32 queries from HBM: two lanes of one 128-B line each (19.4 vs 18.3 G/s at 2^28)
+    if (G == 32 && !insert && !small && t->probe_mode == 0 && t->align == 16) v = 16;
   }
-  v = std::min(v, std::min(G, t->spl == 16 ? 16 : 8));
+  v = std::min(v, std::min(G, (t->spl == 16 || v == 16) ? 16 : 8));
   return v;
 }
 inline int choose_k(const wd_table* t, const Shard& s, int G, int V, bool insert) {
@@ -350,10 +352,20 @@ wd_status_t launch_probe_g(wd_table* t, Shard& s, const In& in, const Out& out, 
   // lanes of 64 B and two keys in flight win (alpha 0.97 / 0.98 / 0.99: 17.7 / 15.9 / 13.4
   // vs 17.1 / 16.2 / 14.9 G/s).  Not for queries from HBM: one lane per 128-B line drops them
   // to 9 G/s.
-  if constexpr (G == 16 && INSERT && std::is_same_v<In, wd::InBucket>)
-    if (t->spl == 0 && t->kif == 0 && t->probe_mode == 0 && t->align == 16 &&
-        double(t->est_size) <= 0.975 * double(s.cap))
-      return launch_gv<G, 16, INSERT>(t, s, in, out, n_hint, st, 1);
+  // The same holds for every |g| >= 4 in the sliced launches (a good part of each slice is in
+  // L2, where one lane per window is the instruction-lean choice, as for small tables):
+  // |g| = 4 V = 4, K = 2: 16.4 -> 19.9; |g| = 8 V = 8, K = 2: 18.8 -> 21.1; |g| = 32 V = 16,
+  // K = 1 (two lanes of one line each): 12.9 -> 14.1 G inserts/s (tools/gpu_vk_all.sh,
+  // profiles/r02/vk_all.jsonl, 2^28, alpha 0.95).
+  if constexpr (G >= 4 && INSERT && std::is_same_v<In, wd::InBucket>)
+    if (t->spl == 0 && t->kif == 0 && t->probe_mode == 0 &&
+        double(t->est_size) <= 0.975 * double(s.cap)) {
+      if constexpr (G >= 16) {
+        if (t->align == 16) return launch_gv<G, 16, INSERT>(t, s, in, out, n_hint, st, 1);
+      } else {
+        return launch_gv<G, G, INSERT>(t, s, in, out, n_hint, st, 2);
+      }
+    }
   const int v = choose_v(t, s, G, INSERT), k = choose_k(t, s, G, v, INSERT);
   if constexpr (G >= 16)
     if (v == 16) return launch_gv<G, 16, INSERT>(t, s, in, out, n_hint, st, k);
