@@ -222,9 +222,9 @@ typedef enum {
                                 (> 1 GB where the span read-ahead applies) and calls of
                                 >= 2^26 pairs, the power of two that makes a slice <= 80 MB
                                 for |g| = 16 on line-aligned tables (32 for config 2's
-                                2.3 GB) or <= 160 MB otherwise, at most 32, and off when a
+                                2.3 GB) or <= 160 MB otherwise, at most 128, and off when a
                                 slice would exceed 300 MB (measured slower);
-                                1: off; 2..32: that many slices.  Uses 8 B of scratch per pair,
+                                1: off; 2..128: that many slices.  Uses 8 B of scratch per pair,
                                 two buffers of at most 2^28 pairs (grouping of the next chunk
                                 overlaps the probing of this one), kept for the table's lifetime
                                 (stream-ordered allocation); in auto mode a failed scratch

@@ -601,7 +601,7 @@ int choose_slices(const wd_table* t, const Shard& s, int op, uint64_t n) {
   // otherwise (|g| = 4: 16 slices 15.5, 32 slices 13.4 G/s)
   const double target = (t->G_used == 16 && t->align == 16) ? 80e6 : 160e6;
   int nbk = 2;
-  while (nbk < wd::kMaxShards && tb / nbk > target) nbk *= 2;
+  while (nbk < wd::kMaxSlices && tb / nbk > target) nbk *= 2;
   if (tb / nbk > 300e6) return 1;
   return nbk;
 }
@@ -658,27 +658,32 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
     }
     s.sl_cap[b] = cap;
   }
-  if (!s.sl_meta) CK(cudaMalloc(&s.sl_meta, 2 * 97 * sizeof(unsigned long long)));
+  constexpr int kMeta = 3 * wd::kMaxSlices + 1;   // counts | bounds (+1) | cursor
+  if (!s.sl_meta) CK(cudaMalloc(&s.sl_meta, 2 * kMeta * sizeof(unsigned long long)));
   // the grouping stream starts after everything st has so far (inputs, scratch allocation)
   CK(cudaEventRecord(s.sl_fork, st));
   CK(cudaStreamWaitEvent(s.s_group, s.sl_fork, 0));
-  const int ms_grid_cap = t->sm_count * blocks_per_sm(wd::multisplit_kernel<true>);
+  // the multisplit instance with the fewest destination slots that fits nbk (its cost grows
+  // with them: 32 slices through the 128-slot instance took 3.1 instead of 1.95 ms per 2^28)
+  auto ms_kern = nbk <= 32 ? wd::multisplit_kernel<true, 32>
+                           : nbk <= 64 ? wd::multisplit_kernel<true, 64> : wd::multisplit_kernel<true, wd::kMaxSlices>;
+  const int ms_grid_cap = t->sm_count * blocks_per_sm(ms_kern);
   const uint64_t nchunks = (io.n + kChunkPairs - 1) / kChunkPairs;
   auto group = [&](uint64_t c) -> wd_status_t {   // on s_group, into buffer c % 2
     const int b = int(c % 2);
     const uint64_t off = c * kChunkPairs, cnt = std::min(kChunkPairs, io.n - off);
-    unsigned long long* counts = s.sl_meta + b * 97;
-    unsigned long long* bounds = counts + 32;
-    unsigned long long* cursor = counts + 65;
+    unsigned long long* counts = s.sl_meta + b * kMeta;
+    unsigned long long* bounds = counts + wd::kMaxSlices;
+    unsigned long long* cursor = counts + 2 * wd::kMaxSlices + 1;
     if (c >= 2) CK(cudaStreamWaitEvent(s.s_group, s.sl_probed[b], 0));   // probes of c - 2 done
     const Ph pg = ph_begin(t, wd::PH_GROUP, s.device, s.s_group);
     CK(cudaMemsetAsync(counts, 0, nbk * sizeof(unsigned long long), s.s_group));
     wd::slice_hist_kernel<<<t->sm_count * 4, wd::kBlock, 0, s.s_group>>>(io.keys + off, cnt, nbk, s.hseed, counts);
     wd::slice_scan_kernel<<<1, 32, 0, s.s_group>>>(counts, nbk, bounds, cursor);
-    wd::DstPtrs dst{};
-    for (int d = 0; d < nbk; ++d) dst.p[d] = s.sl_buf[b];
+    wd::DstPtrs dst{};                               // one buffer, slice j at bounds[j]
+    for (int d = 0; d < wd::kMaxShards; ++d) dst.p[d] = s.sl_buf[b];
     const uint64_t tiles = (cnt + wd::kMsTile - 1) / wd::kMsTile;
-    wd::multisplit_kernel<true><<<int(std::min<uint64_t>(tiles, uint64_t(ms_grid_cap))), wd::kBlock, 0, s.s_group>>>(
+    ms_kern<<<int(std::min<uint64_t>(tiles, uint64_t(ms_grid_cap))), wd::kBlock, 0, s.s_group>>>(
         io.keys + off, io.vals + off, cnt, dst, cursor, nullptr, nbk, s.hseed, 0, cnt, s.counters);
     CK(cudaGetLastError());
     t->launches += 3;
@@ -689,7 +694,7 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
   auto probe = [&](uint64_t c) -> wd_status_t {   // on st
     const int b = int(c % 2);
     const uint64_t off = c * kChunkPairs, cnt = std::min(kChunkPairs, io.n - off);
-    const unsigned long long* bounds = s.sl_meta + b * 97 + 32;
+    const unsigned long long* bounds = s.sl_meta + b * kMeta + wd::kMaxSlices;
     CK(cudaStreamWaitEvent(st, s.sl_grouped[b], 0));
     const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, st);
     for (int j = 0; j < nbk; ++j)
@@ -1855,7 +1860,7 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       t->span = int(v);
       return WD_OK;
     case WD_OPT_SLICES:
-      if (v < 0 || v > wd::kMaxShards) return fail(WD_ERR_INVALID_ARG, "slices %lld", (long long)v);
+      if (v < 0 || v > wd::kMaxSlices) return fail(WD_ERR_INVALID_ARG, "slices %lld", (long long)v);
       t->slices = int(v);
       return WD_OK;
     case WD_OPT_PHASE_TIMING:
