@@ -446,7 +446,7 @@ def test_span_read_ahead(wd, G, span):
 
 
 @pytest.mark.parametrize("G", [4, 16])
-@pytest.mark.parametrize("slices", [1, 2, 16, 32])
+@pytest.mark.parametrize("slices", [1, 2, 16, 32, 64, 128])
 def test_slice_grouped_insert(wd, G, slices):
     # WD_OPT_SLICES: a bulk insert grouped by table slice of the first region and inserted
     # with one launch per slice.  Unique keys: exact map; duplicates with a reserved key:
