@@ -256,7 +256,8 @@ typedef enum {
                                 1 = after an insert call that left keys behind (Line 26) while
                                 live keys + those keys still fit the capacity (e.g. tombstones
                                 fill the probe sequences), rebuild with a new seed and re-insert
-                                them (up to 4 times).  Makes wd_insert synchronous.  0
+                                them (up to 4 times).  Makes wd_insert synchronous; applies
+                                to whole-table wd_insert calls (not the _sharded ones).  0
                                 (default): off, the sticky WD_ERR_TABLE_FULL is reported.
                                 Single-process tables only (not rank mode). */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */

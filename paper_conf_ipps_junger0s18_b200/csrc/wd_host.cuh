@@ -15,6 +15,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <type_traits>
+#include <mutex>
 #include <unordered_map>
 #include <vector>
 
@@ -209,16 +210,17 @@ inline PtrKind classify(const void* p, int* dev) {
   return PK_PAGEABLE;
 }
 
+// resident blocks per SM of a kernel (occupancy API), cached; tables may be used from
+// several host threads (one thread per table), so the cache is guarded
 template <class K>
-int blocks_per_sm(K kern, size_t dyn_smem = 0) {
+int blocks_per_sm(K kern) {
   static std::unordered_map<const void*, int> cache;
+  static std::mutex mu;
+  std::lock_guard<std::mutex> lk(mu);
   auto it = cache.find((const void*)kern);
   if (it != cache.end()) return it->second;
   int nb = 0;
-  if (dyn_smem > 48 * 1024 &&
-      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(dyn_smem)) != cudaSuccess)
-    cudaGetLastError();
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, wd::kBlock, dyn_smem) != cudaSuccess) {
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kern, wd::kBlock, 0) != cudaSuccess) {
     cudaGetLastError();
     nb = 1;
   }
@@ -234,7 +236,6 @@ template <int G, int V, int K, bool INSERT, class In, class Out, int S = 1>
 wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                            cudaStream_t st) {
   auto kern = wd::probe_kernel<G, V, K, INSERT, In, Out, S>;
-  const size_t smem = 0;
   // C4': default p_max = nb — eq. 3 then visits every region, so an insert fails only when
   // no slot is free (a fixed 1024 is exceeded at alpha = 0.999 even sequentially).
   const uint32_t pmax = t->pmax > 0 ? static_cast<uint32_t>(t->pmax) : static_cast<uint32_t>(s.nb);
@@ -245,11 +246,11 @@ wd_status_t launch_probe_k(wd_table* t, Shard& s, const In& in, const Out& out, 
     block = wd::kBlock;
     const uint64_t keys_per_block = uint64_t(wd::kBlock / 32) * K * (32 / (G / V));
     const uint64_t need = std::max<uint64_t>(1, (n_hint + keys_per_block - 1) / keys_per_block);
-    grid = static_cast<int>(std::min<uint64_t>(need, uint64_t(t->sm_count) * blocks_per_sm(kern, smem)));
+    grid = static_cast<int>(std::min<uint64_t>(need, uint64_t(t->sm_count) * blocks_per_sm(kern)));
     static const int cap_env = getenv("WD_MAX_BLOCKS") ? atoi(getenv("WD_MAX_BLOCKS")) : 0;
     if (cap_env > 0) grid = std::min(grid, cap_env);   // measurement hook (tools/)
   }
-  kern<<<grid, block, smem, st>>>(tv, in, out, s.counters, t->serial);
+  kern<<<grid, block, 0, st>>>(tv, in, out, s.counters, t->serial);
   CK(cudaGetLastError());
   t->launches++;
   return WD_OK;
