@@ -875,6 +875,29 @@ def run_sweep(args, wd, gg, torch):
     return out
 
 
+def l2_roofline(G, ins, qry):
+    """Config 1's table (8.8 MB) is L2-resident: its ceiling is this B200's random L2 rate
+    for the kernels' own pattern (tools/randbench 0.0088 -> profiles/ceilings.json "l2_8.8MB"):
+    an insert = (L - 1) window reads + one read-then-CAS, a query = L window reads, L from the
+    oracle replay (hits; misses for the absent half of the queries)."""
+    cf = os.path.join(ROOT, "profiles", "ceilings.json")
+    if not os.path.exists(cf):
+        return None
+    c = json.load(open(cf)).get("l2_8.8MB")
+    wb = str(min(8 * G, 256))
+    if not c or wb not in c["read"] or wb not in c["casw"]:
+        return None
+    pc = probe_cost(0.95, G)
+    R, C = c["read"][wb], c["casw"][wb]
+    ins_ceiling = 1.0 / ((pc["ins_windows"] - 1) / R + 1 / C)
+    q_ceiling = R / (0.5 * pc["hit_windows"] + 0.5 * pc["miss_windows"])
+    return {"insert_ceiling_gops": ins_ceiling, "insert_frac": ins / ins_ceiling,
+            "query_ceiling_gops": q_ceiling, "query_frac": qry / q_ceiling,
+            "rates_Gwin_s": {"read": R, "casw": C}, "windows": {
+                "insert": pc["ins_windows"], "hit": pc["hit_windows"], "miss": pc["miss_windows"]},
+            "source": "profiles/ceilings.json l2_8.8MB"}
+
+
 def run_config1(wd, gg, torch):
     """BASELINE config 1: 2^20 unique pairs at alpha 0.95 (an 8.8 MB, L2-resident table),
     then all 2^20 keys + 2^20 absent keys queried (interleaved); |g| = 4 as configured,
@@ -902,10 +925,11 @@ def run_config1(wd, gg, torch):
                     ti.append(a.elapsed_time(b))
                     tq.append(b.elapsed_time(c))
             assert t.sync() == 0 and t.size() == n and int(fout.sum().item()) == n
+            ins = n / (sum(ti) / len(ti)) / 1e6
+            qry = 2 * n / (sum(tq) / len(tq)) / 1e6
             out.append({"sweep": "config1", "alpha": 0.95, "G": G, "keys": n, "queries": 2 * n,
-                        "table_MB": t.capacity() * 8 / 1e6,
-                        "insert_gops": n / (sum(ti) / len(ti)) / 1e6,
-                        "query_gops": 2 * n / (sum(tq) / len(tq)) / 1e6})
+                        "table_MB": t.capacity() * 8 / 1e6, "insert_gops": ins, "query_gops": qry,
+                        "l2_roofline": l2_roofline(G, ins, qry)})
     return out
 
 

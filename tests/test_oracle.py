@@ -494,3 +494,51 @@ def test_replay_rebuild_drops_tombstones():
     # a distinct seed is a distinct probe sequence ("distinct hash function")
     assert any(oracle.Replay.base(int(k), 0, c, 0x1234567) != oracle.Replay.base(int(k), 0, c)
                for k in keys[:20])
+
+
+def test_partition_power_of_two_is_top_bits():
+    # P:99 / C15 special case: for m = 2^b, floor(fmix32(k + s) m / 2^32) is the top b bits of
+    # fmix32(k + s) — an identity, checked through the separately pinned fmix32 (Murmur3
+    # vectors); a wrong hash, a missing seed or a wrong product would fail it
+    rng = np.random.default_rng(12)
+    keys = rng.integers(0, 2**32 - 1, 200_000, dtype=np.uint64).astype(np.uint32)
+    for b in (1, 2, 3, 5):
+        for seed in (0, 0x9E3779B9, 12345):
+            d = oracle.partition(keys, 1 << b, seed)
+            h = oracle.fmix32_many((keys.astype(np.uint64) + seed) & 0xFFFFFFFF)
+            assert np.array_equal(d, (h >> np.uint32(32 - b)).astype(d.dtype))
+
+
+def test_table_scans_place_every_key_once():
+    # P:117 transposition simulated end to end with the oracle's multisplit (an independent
+    # layout: perm) and table_scans: source g's bucket for owner p starts at send_off[g][p] in
+    # g's multisplit output and lands at recv_off[p][g] in p's receive buffer.  Every owner
+    # must receive exactly its keys, each once, grouped by source in source order.
+    rng = np.random.default_rng(21)
+    for m in (2, 3, 4, 8):
+        seed = 77
+        srcs = [rng.integers(0, 2**32 - 1, int(rng.integers(0, 3000)), dtype=np.uint64).astype(np.uint32)
+                for _ in range(m)]
+        T = np.zeros((m, m), np.uint64)
+        outs = []
+        for g, k in enumerate(srcs):
+            counts, perm = oracle.multisplit(k, m, seed)
+            T[g] = counts
+            out = np.empty_like(k)
+            out[perm.astype(np.int64)] = k
+            outs.append(out)
+        so, ro = oracle.table_scans(T)
+        for p in range(m):
+            recv = np.full(int(T[:, p].sum()), 0xFFFFFFFF, np.uint32)
+            filled = np.zeros(recv.size, bool)
+            for g in range(m):
+                c = int(T[g, p])
+                blk = outs[g][int(so[g, p]): int(so[g, p]) + c]
+                assert np.all(oracle.partition(blk, m, seed) == p)          # right bucket
+                dst = slice(int(ro[p, g]), int(ro[p, g]) + c)
+                assert not filled[dst].any()                                  # disjoint
+                recv[dst] = blk
+                filled[dst] = True
+            assert filled.all()
+            want = np.concatenate([k[oracle.partition(k, m, seed) == p] for k in srcs])
+            assert np.array_equal(recv, want)                                 # all, in order
