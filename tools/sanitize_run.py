@@ -31,6 +31,17 @@ with wd.Table(capacity_for(n, 0.9), 1, 8, batch=3000) as t:
 with wd.Table(capacity_for(n, 0.9), 1, 16) as t:
     t.set_option(wd.WD_OPT_SLOTS_PER_LANE, 16)
     check(*gpu_roundtrip(t, keys, vals, q))
+for nbk, G in ((64, 16), (128, 4), (32, 8)):       # the 64- / 128-slot multisplit instances
+    with wd.Table(capacity_for(n, 0.9), 1, G) as t:
+        t.set_option(wd.WD_OPT_SLICES, nbk)
+        check(*gpu_roundtrip(t, keys, vals, q))
+with wd.Table(capacity_for(n, 0.9), 1, 8) as t:  # automatic rebuild after tombstones fill it
+    t.set_option(wd.WD_OPT_AUTO_REBUILD, 1)
+    t.insert(torch.from_numpy(keys.view(np.int32)).cuda(), torch.from_numpy(vals.view(np.int32)).cuda())
+    t.erase(torch.from_numpy(keys[: n // 2].view(np.int32)).cuda())
+    more = wdgen.unique_keys(n // 2, 1, start=n)
+    t.insert(torch.from_numpy(more.view(np.int32)).cuda(), torch.from_numpy(wdgen.values(n // 2, 3).view(np.int32)).cuda())
+    assert t.sync() == 0 and t.size() == n
 with wd.Table(capacity_for(n, 0.9), group_size=8, loopback_shards=3, batch=3000, exchange=1) as t:
     check(*gpu_roundtrip(t, keys, vals, q))
     er = t.erase(torch.from_numpy(q[: n // 2].view(np.int32)).cuda())
