@@ -658,33 +658,40 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
     }
     s.sl_cap[b] = cap;
   }
-  constexpr int kMeta = 3 * wd::kMaxSlices + 1;   // counts | bounds (+1) | cursor
+  // the multisplit instance with the fewest destination slots that fits nbk, in segment
+  // mode: grid = one block per SM slot, block b groups the contiguous segment
+  // [b L, (b + 1) L) of the chunk (L a multiple of the tile)
+  auto ms_kern = nbk <= 32 ? wd::multisplit_kernel<true, 1, true, true>
+                           : nbk <= 64 ? wd::multisplit_kernel<true, 2, true, true>
+                                       : wd::multisplit_kernel<true, wd::kMaxSlices / 32, true, true>;
+  const int S = t->sm_count * blocks_per_sm(ms_kern);
+  const int S_max = t->sm_count * std::max({blocks_per_sm(wd::multisplit_kernel<true, 1, true, true>),
+                                            blocks_per_sm(wd::multisplit_kernel<true, 2, true, true>),
+                                            blocks_per_sm(wd::multisplit_kernel<true, wd::kMaxSlices / 32, true, true>)});
+  // per buffer: bounds (kMaxSlices + 1) | cursor (kMaxSlices) | seg_off (S_max x kMaxSlices)
+  // | seg counts (S_max x kMaxSlices u32, in u64 words)
+  const uint64_t kMeta = 2 * wd::kMaxSlices + 1 + uint64_t(S_max) * wd::kMaxSlices * 3 / 2 + 1;
   if (!s.sl_meta) CK(cudaMalloc(&s.sl_meta, 2 * kMeta * sizeof(unsigned long long)));
   // the grouping stream starts after everything st has so far (inputs, scratch allocation)
   CK(cudaEventRecord(s.sl_fork, st));
   CK(cudaStreamWaitEvent(s.s_group, s.sl_fork, 0));
-  // the multisplit instance with the fewest destination slots that fits nbk (its cost grows
-  // with them: 32 slices through the 128-slot instance took 3.1 instead of 1.95 ms per 2^28)
-  auto ms_kern = nbk <= 32 ? wd::multisplit_kernel<true, 32>
-                           : nbk <= 64 ? wd::multisplit_kernel<true, 64> : wd::multisplit_kernel<true, wd::kMaxSlices>;
-  const int ms_grid_cap = t->sm_count * blocks_per_sm(ms_kern);
   const uint64_t nchunks = (io.n + kChunkPairs - 1) / kChunkPairs;
   auto group = [&](uint64_t c) -> wd_status_t {   // on s_group, into buffer c % 2
     const int b = int(c % 2);
     const uint64_t off = c * kChunkPairs, cnt = std::min(kChunkPairs, io.n - off);
-    unsigned long long* counts = s.sl_meta + b * kMeta;
-    unsigned long long* bounds = counts + wd::kMaxSlices;
-    unsigned long long* cursor = counts + 2 * wd::kMaxSlices + 1;
+    unsigned long long* bounds = s.sl_meta + b * kMeta;
+    unsigned long long* cursor = bounds + wd::kMaxSlices + 1;
+    unsigned long long* seg_off = cursor + wd::kMaxSlices;
+    unsigned int* seg_cnt = reinterpret_cast<unsigned int*>(seg_off + uint64_t(S_max) * wd::kMaxSlices);
     if (c >= 2) CK(cudaStreamWaitEvent(s.s_group, s.sl_probed[b], 0));   // probes of c - 2 done
     const Ph pg = ph_begin(t, wd::PH_GROUP, s.device, s.s_group);
-    CK(cudaMemsetAsync(counts, 0, nbk * sizeof(unsigned long long), s.s_group));
-    wd::slice_hist_kernel<<<t->sm_count * 4, wd::kBlock, 0, s.s_group>>>(io.keys + off, cnt, nbk, s.hseed, counts);
-    wd::slice_scan_kernel<<<1, 32, 0, s.s_group>>>(counts, nbk, bounds, cursor);
+    const uint64_t L = ((cnt + S - 1) / S + wd::kMs2Tile - 1) / wd::kMs2Tile * wd::kMs2Tile;
+    wd::seg_hist_kernel<<<S, wd::kBlock, 0, s.s_group>>>(io.keys + off, cnt, L, nbk, s.hseed, seg_cnt);
+    wd::seg_scan_kernel<<<1, 1024, 0, s.s_group>>>(seg_cnt, S, nbk, bounds, cursor, seg_off);
     wd::DstPtrs dst{};                               // one buffer, slice j at bounds[j]
-    for (int d = 0; d < wd::kMaxShards; ++d) dst.p[d] = s.sl_buf[b];
-    const uint64_t tiles = (cnt + wd::kMsTile - 1) / wd::kMsTile;
-    ms_kern<<<int(std::min<uint64_t>(tiles, uint64_t(ms_grid_cap))), wd::kBlock, 0, s.s_group>>>(
-        io.keys + off, io.vals + off, cnt, dst, cursor, nullptr, nbk, s.hseed, 0, cnt, s.counters);
+    dst.p[0] = s.sl_buf[b];
+    ms_kern<<<S, wd::kBlock, 0, s.s_group>>>(io.keys + off, io.vals + off, cnt, dst, nullptr, seg_off, L,
+                                             nullptr, nbk, s.hseed, cnt, s.counters);
     CK(cudaGetLastError());
     t->launches += 3;
     ph_end(t, pg);
@@ -694,7 +701,7 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
   auto probe = [&](uint64_t c) -> wd_status_t {   // on st
     const int b = int(c % 2);
     const uint64_t off = c * kChunkPairs, cnt = std::min(kChunkPairs, io.n - off);
-    const unsigned long long* bounds = s.sl_meta + b * kMeta + wd::kMaxSlices;
+    const unsigned long long* bounds = s.sl_meta + b * kMeta;
     CK(cudaStreamWaitEvent(st, s.sl_grouped[b], 0));
     const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, st);
     for (int j = 0; j < nbk; ++j)
@@ -918,17 +925,16 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
       else dst.p[d] = reinterpret_cast<uint32_t*>(t->peers[d].recv[slot]) + uint64_t(s.id) * B;
     }
     // every resident block of the SM (occupancy API): more tiles in flight per SM
-    const uint64_t tiles = (cnt + wd::kMsTile - 1) / wd::kMsTile;
-    const int per_sm = insert ? blocks_per_sm(wd::multisplit_kernel<true>)
-                              : blocks_per_sm(wd::multisplit_kernel<false>);
-    const int grid = int(std::min<uint64_t>(tiles, uint64_t(t->sm_count) * per_sm));
-    if (insert)
-      wd::multisplit_kernel<true><<<grid, wd::kBlock, 0, s.s_main>>>(
-          dk, dv, cnt, dst, s.cursor[slot], nullptr, m, t->pseed, t->pmode, B, s.counters);
-    else
-      wd::multisplit_kernel<false><<<grid, wd::kBlock, 0, s.s_main>>>(
-          dk, nullptr, cnt, dst, s.cursor[slot], s.pos[slot], m, t->pseed, t->pmode, B,
-          s.counters);
+    // cursor mode (the owners read their column of T from the cursors), p(k) of C15 or
+    // Fig. 4's k mod m (WD_OPT_PART_MODE)
+    auto kern = insert ? (t->pmode == 1 ? wd::multisplit_kernel<true, 1, false, false, 1>
+                                        : wd::multisplit_kernel<true, 1, false, false, 0>)
+                       : (t->pmode == 1 ? wd::multisplit_kernel<false, 1, false, false, 1>
+                                        : wd::multisplit_kernel<false, 1, false, false, 0>);
+    const uint64_t tiles = (cnt + wd::kMs2Tile - 1) / wd::kMs2Tile;
+    const int grid = int(std::min<uint64_t>(tiles, uint64_t(t->sm_count) * blocks_per_sm(kern)));
+    kern<<<grid, wd::kBlock, 0, s.s_main>>>(dk, insert ? dv : nullptr, cnt, dst, s.cursor[slot], nullptr, 0,
+                                             insert ? nullptr : s.pos[slot], m, t->pseed, B, s.counters);
     CK(cudaGetLastError());
     t->launches++;
     return WD_OK;

@@ -328,7 +328,6 @@ inline int choose_v(const wd_table* t, const Shard& s, int G, bool insert) {
 }
 inline int choose_k(const wd_table* t, const Shard& s, int G, int V, bool insert) {
   if (t->kif) return t->kif;
-  const bool small = s.cap * sizeof(unsigned long long) <= (64ull << 20);
   // |g| = 1 inserts into tables > 1 GB run slice-grouped (no span read-ahead): K = 4
   // (2^28, alpha 0.95: 7.5 -> 9.7 G/s); queries and smaller tables keep K = 8 with the span.
   if (V == 1) return (G == 1 && insert && double(s.cap) * 8 > 1.0e9) ? 4 : (G <= 4 ? 8 : 4);
