@@ -704,6 +704,9 @@ wd_status_t slice_insert(wd_table* t, Shard& s, const IO& io, int nbk, cudaStrea
     const unsigned long long* bounds = s.sl_meta + b * kMeta;
     CK(cudaStreamWaitEvent(st, s.sl_grouped[b], 0));
     const Ph pp = ph_begin(t, wd::PH_PROBE, s.device, st);
+    // (programmatic dependent launch of slice j + 1 into slice j's tail was measured slower:
+    // 10.4 -> 11.1 ms for the 32 launches, two slices' working sets share the L2 —
+    // profiles/r02/pdl_negative.md)
     for (int j = 0; j < nbk; ++j)
       TRY(launch_probe<true>(t, s, wd::InBucket{s.sl_buf[b], bounds, j, j + 1}, wd::OutNone{},
                              cnt / nbk + 1, st));
