@@ -847,24 +847,30 @@ def run_sweep(args, wd, gg, torch):
     for alpha in (0.8, 0.9, 0.95, 0.99):
         for G in (1, 2, 4, 8, 16, 32):
             with wd.Table(int(math.ceil(n / alpha)), 1, G) as t:
-                ti, tq = [], []
+                ti, tq, tauto = [], [], []
                 for it in range(4):
-                    a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+                    a, b, c, d = (torch.cuda.Event(enable_timing=True) for _ in range(4))
                     t.clear(s)
                     a.record(s)
                     t.insert(keys, vals, s)
                     b.record(s)
+                    t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)     # the paper's: same |g|
                     t.retrieve(keys, vout, fout, s)
                     c.record(s)
+                    t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, -1)    # the library default (auto)
+                    t.retrieve(keys, vout, fout, s)
+                    d.record(s)
                     torch.cuda.synchronize()
                     if it:
                         ti.append(a.elapsed_time(b))
                         tq.append(b.elapsed_time(c))
+                        tauto.append(c.elapsed_time(d))
                 assert t.sync() == 0
                 pc = probe_cost(alpha, G)
                 ims, qms = sum(ti) / len(ti), sum(tq) / len(tq)
                 out.append({"sweep": "config2", "alpha": alpha, "G": G,
                             "insert_gops": n / ims / 1e6, "query_gops": n / qms / 1e6,
+                            "query_gops_auto": n / (sum(tauto) / len(tauto)) / 1e6,
                             "insert_frac": n * (40 + 32 * pc["ins_sectors"]) / (ims * 1e-3) / 1e9 / hbm,
                             "query_frac": n * (9 + 32 * pc["hit_sectors"]) / (qms * 1e-3) / 1e9 / hbm})
     out += run_config1(wd, gg, torch)
@@ -909,8 +915,9 @@ def run_config1(wd, gg, torch):
     vout = torch.empty(2 * n, dtype=torch.int32, device="cuda")
     fout = torch.empty(2 * n, dtype=torch.uint8, device="cuda")
     s = torch.cuda.current_stream()
-    for G in (4, 8, 16):
+    for G, qg in ((4, 0), (8, 0), (16, 0), (4, -1), (8, -1)):
         with wd.Table(int(math.ceil(n / 0.95)), 1, G) as t:
+            t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)   # 0: the paper's (queries with |g|)
             ti, tq = [], []
             for it in range(11):
                 a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
@@ -927,7 +934,7 @@ def run_config1(wd, gg, torch):
             assert t.sync() == 0 and t.size() == n and int(fout.sum().item()) == n
             ins = n / (sum(ti) / len(ti)) / 1e6
             qry = 2 * n / (sum(tq) / len(tq)) / 1e6
-            out.append({"sweep": "config1", "alpha": 0.95, "G": G, "keys": n, "queries": 2 * n,
+            out.append({"sweep": "config1", "alpha": 0.95, "G": G, "query_G": "auto" if qg < 0 else G, "keys": n, "queries": 2 * n,
                         "table_MB": t.capacity() * 8 / 1e6, "insert_gops": ins, "query_gops": qry,
                         "l2_roofline": l2_roofline(G, ins, qry)})
     return out
@@ -948,7 +955,10 @@ def run_mix(wd, gg, torch, keys, vals, log2n):
     for G in (4, 8, 16):
         with wd.Table(int(math.ceil(n / 0.95)), 1, G) as t:
             t.insert(keys, vals, s)
-            for h in (0.0, 0.5, 1.0):
+            for h, qg in ((0.0, 0), (0.5, 0), (1.0, 0), (0.0, -1), (0.5, -1), (1.0, -1)):
+                if qg < 0 and G == 16:
+                    continue
+                t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)   # 0: the paper's (queries with |g|)
                 gg.mixed_queries(n, n, h, KEY_SEED, out=q, hits=hits)
                 ts = []
                 for it in range(4):
@@ -963,10 +973,11 @@ def run_mix(wd, gg, torch, keys, vals, log2n):
                 ms = sum(ts) / len(ts)
                 pc = probe_cost(0.95, G)
                 S = h * pc["hit_sectors"] + (1 - h) * pc["miss_sectors"]
-                out.append({"sweep": "config4_mix_1gpu", "alpha": 0.95, "G": G, "hit_frac": h,
+                # the replay's sector counts are for windows of the table's |g| (qg = 0)
+                out.append({"sweep": "config4_mix_1gpu", "alpha": 0.95, "G": G, "query_G": "auto" if qg < 0 else G, "hit_frac": h,
                             "table_keys": n, "queries": n, "query_gops": n / ms / 1e6,
-                            "sectors_per_query": S,
-                            "query_frac": n * (9 + 32 * S) / (ms * 1e-3) / 1e9 / hbm})
+                            "sectors_per_query": S if not qg else None,
+                            "query_frac": n * (9 + 32 * S) / (ms * 1e-3) / 1e9 / hbm if not qg else None})
     return out
 
 

@@ -260,6 +260,17 @@ typedef enum {
                                 to whole-table wd_insert calls (not the _sharded ones).  0
                                 (default): off, the sticky WD_ERR_TABLE_FULL is reported.
                                 Single-process tables only (not rank mode). */
+    WD_OPT_QUERY_GROUP_SIZE = 16, /* |g| of wd_retrieve / wd_erase calls.  P:89: the probe
+                                sequence, hence every result, is the same for any |g| (a key
+                                sits at the leftmost empty slot of its sequence, so no empty
+                                slot precedes it for any window size).  -1 (default): auto,
+                                by region alignment and load: 16 (one 128-byte line) on A = 16
+                                tables and above a projected load of 0.93, else 8.  Measured
+                                on B200 (profiles/r02/sweep_r02o.jsonl, query_group.jsonl;
+                                2^28 keys): alpha 0.95 hits on |g| = 1 / 2 / 4 / 32 tables
+                                7.0 / 10.4 / 17.6 / 19.0 -> 24.2 / 24.2 / 24.3 / 26.6 G/s,
+                                misses on |g| = 4 2.9 -> 7.9 G/s.  0: the inserts' |g| (the
+                                paper's setting); else 1..32. */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -1262,12 +1262,21 @@ wd_status_t classify_io(wd_table* t, bool insert, IO& io, int shard) {
 // step): |g| = 8 is fastest up to alpha 0.9, |g| = 16 from 0.95 on (and for misses at any
 // load).  The load used is the projected one after this call, from a host-side upper
 // estimate of the size (no synchronisation).
+// Queries and erases use WD_OPT_QUERY_GROUP_SIZE: the same results for any |g|.  Auto
+// (default): the layout, hence the query cost, depends only on the load and the region
+// alignment A, not on the |g| the keys were inserted with; measured on B200
+// (profiles/r02/sweep_r02o.jsonl, 2^28 keys, hits): A = 16 tables: |g| 16 (one line per
+// window) at every load; A = 4 tables: |g| 8 up to a load of 0.93 (alpha 0.8 / 0.9: 32.2 /
+// 28.0 G/s against 27.1 / 26.1 with 16-slot windows, which straddle two lines there), |g|
+// 16 above (0.95 / 0.99: 24.3 / 20.2 against 24.0 / 18.2); misses favour 16 at any load.
 void pick_group_size(wd_table* t, int op, uint64_t n) {
-  if (t->G == 0) {
-    const double cap = double(wd_capacity(t));
-    const double est = double(t->est_size) + (op == OP_INSERT ? double(n) : 0.0);
-    t->G_used = (est / cap > 0.93) ? 16 : 8;
-  }
+  const double cap = double(wd_capacity(t));
+  const double est = double(t->est_size) + (op == OP_INSERT ? double(n) : 0.0);
+  const bool high = est / cap > 0.93;
+  t->G_ins = t->G ? t->G : (high ? 16 : 8);
+  if (op == OP_INSERT || t->qg == 0) t->G_used = t->G_ins;
+  else if (t->qg > 0) t->G_used = t->qg;
+  else t->G_used = (t->align >= 16 || high) ? 16 : 8;
   if (op == OP_INSERT) t->est_size = std::min<uint64_t>(t->est_size + n, wd_capacity(t));
 }
 
@@ -1438,7 +1447,7 @@ wd_table* create_common(uint64_t capacity, int mode, int m, int group_size) {
   t->mode = mode;
   t->m = m;
   t->G = group_size;
-  t->G_used = group_size ? group_size : 8;
+  t->G_used = t->G_ins = group_size ? group_size : 8;
   t->align = wd::region_align_for(group_size);   // reading C2': fixed for the table's life
   return t;
 }
@@ -1830,7 +1839,12 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
       if (v != 0 && v != 1 && v != 2 && v != 4 && v != 8 && v != 16 && v != 32)
         return fail(WD_ERR_INVALID_ARG, "group size %lld", (long long)v);
       t->G = int(v);
-      if (v) t->G_used = int(v);
+      if (v) t->G_used = t->G_ins = int(v);
+      return WD_OK;
+    case WD_OPT_QUERY_GROUP_SIZE:
+      if (v != -1 && v != 0 && v != 1 && v != 2 && v != 4 && v != 8 && v != 16 && v != 32)
+        return fail(WD_ERR_INVALID_ARG, "query group size %lld", (long long)v);
+      t->qg = int(v);
       return WD_OK;
     case WD_OPT_P_MAX:
       if (v < 0 || v > (1 << 26)) return fail(WD_ERR_INVALID_ARG, "p_max %lld", (long long)v);
@@ -1898,6 +1912,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
   switch (opt) {
     case WD_OPT_GROUP_SIZE: return t->G;
     case WD_OPT_GROUP_SIZE_USED: return t->G_used;
+    case WD_OPT_QUERY_GROUP_SIZE: return t->qg;
     case WD_OPT_REGION_ALIGN: return t->align;
     case WD_OPT_P_MAX: return t->pmax;
     case WD_OPT_BATCH: return int64_t(t->batch);

@@ -140,6 +140,8 @@ struct wd_table {
   int rank = 0;       // rank mode: this process's shard id
   int G = 4;          // |g|, or 0 = dynamic by load
   int G_used = 4;     // |g| of the current / last call
+  int G_ins = 4;      // |g| of the last insert (dynamic |g|: by load)
+  int qg = -1;        // |g| of query / erase calls (WD_OPT_QUERY_GROUP_SIZE; -1 auto, 0 G_ins)
   uint32_t align = 4; // A of reading C2': 16 for tables created with |g| >= 16, else 4
   uint64_t est_size = 0;   // host-side upper estimate of the stored keys (no sync needed)
   int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit
@@ -406,7 +408,10 @@ WD_PROBE_COMBOS(WD_PROBE_EXTERN, 32)
 template <bool INSERT, class In, class Out>
 wd_status_t launch_probe(wd_table* t, Shard& s, const In& in, const Out& out, uint64_t n_hint,
                          cudaStream_t st) {
-  switch (t->G_used) {
+  // inserts (including rebuild re-inserts) with the inserts' |g|; queries / erases with the
+  // |g| pick_group_size chose for the call
+  const int G = INSERT ? t->G_ins : t->G_used;
+  switch (G) {
     case 1: return launch_probe_g<1, INSERT>(t, s, in, out, n_hint, st);
     case 2: return launch_probe_g<2, INSERT>(t, s, in, out, n_hint, st);
     case 4: return launch_probe_g<4, INSERT>(t, s, in, out, n_hint, st);
@@ -414,7 +419,7 @@ wd_status_t launch_probe(wd_table* t, Shard& s, const In& in, const Out& out, ui
     case 16: return launch_probe_g<16, INSERT>(t, s, in, out, n_hint, st);
     case 32: return launch_probe_g<32, INSERT>(t, s, in, out, n_hint, st);
   }
-  return fail(WD_ERR_INVALID_ARG, "group size %d not in {1,2,4,8,16,32}", t->G_used);
+  return fail(WD_ERR_INVALID_ARG, "group size %d not in {1,2,4,8,16,32}", G);
 }
 
 }  // namespace wdi

@@ -83,7 +83,9 @@ def test_config2_grid_every_query(env, alpha, G):
         t.insert(keys, vals)
         del vals
         assert t.sync() == 0 and t.size() == n
-        _roundtrip_all(wd, gg, torch, t, n, keys)
+        for qg in (0, -1):          # queries with the table's |g| (the paper's), and the default
+            t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)
+            _roundtrip_all(wd, gg, torch, t, n, keys)
 
 
 def test_config3_single_gpu_every_query(env):

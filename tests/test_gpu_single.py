@@ -30,14 +30,16 @@ def _oracle_answers(keys, vals, queries, dup=False):
 MODES = [(G, 1) for G in GS] + [(G, 2) for G in GS if G <= 8]   # (|g|, probe mode)
 
 
+@pytest.mark.parametrize("qg", [0, -1])
 @pytest.mark.parametrize("G,mode", MODES)
-def test_config1_unique_parity(wd, G, mode):
+def test_config1_unique_parity(wd, G, mode, qg):
     # BASELINE config 1: 2^20 unique keys, load 0.95, all keys + 2^20 absent keys queried
     n, ks, vs = 1 << 20, 101, 202
     keys, vals = wdgen.unique_keys(n, ks), wdgen.values(n, vs)
     q = wdgen.interleaved_queries(n, ks)
     with wd.Table(capacity_for(n, 0.95), 1, G) as t:
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
+        t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)      # 0: queries with the table's |g|
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0
         assert t.size() == n
@@ -66,6 +68,7 @@ def test_alpha_and_keys_in_flight(wd, alpha, kif, mode):
     with wd.Table(capacity_for(n, alpha), 1, 4) as t:
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, kif)
+        t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0 and t.size() == n
     cv, cf = oracle.expected_unique(q, n, 7, 8)
@@ -117,7 +120,7 @@ def test_region_align_is_per_table(wd, Gc, Gi):
         q = wdgen.interleaved_queries(n, 51)
         cv, cf = oracle.expected_unique(q, n, 51, 52)
         for Gq in (1, 4, 16, 32):
-            t.set_option(wd.WD_OPT_GROUP_SIZE, Gq)
+            t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, Gq)
             ov, of = t.retrieve(to_dev(q))
             assert np.array_equal(of.cpu().numpy(), cf) and np.array_equal(from_dev(ov), cv)
 
@@ -133,12 +136,47 @@ def test_cross_group_size(wd, Gi, Gq, mi, mq):
     with wd.Table(capacity_for(n, 0.97), 1, Gi) as t:
         t.set_option(wd.WD_OPT_PROBE_MODE, mi)
         t.insert(to_dev(keys), to_dev(vals))
-        t.set_option(wd.WD_OPT_GROUP_SIZE, Gq)
+        t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, Gq)
         t.set_option(wd.WD_OPT_PROBE_MODE, mq)
         ov, of = t.retrieve(to_dev(q))
         gv, gf = from_dev(ov), of.cpu().numpy()
     cv, cf = oracle.expected_unique(q, n, 9, 9)
     assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
+@pytest.mark.parametrize("G", [1, 2, 4, 8, 16, 32])
+def test_query_group_size(wd, G):
+    # WD_OPT_QUERY_GROUP_SIZE (default -1 = auto): retrieve / erase with a |g| other than the
+    # inserts' — P:89, every result is the same: hits, misses (long chains at alpha 0.97),
+    # erase flags, queries past tombstones, and the values of updated keys
+    n = 120_001
+    keys, vals = wdgen.unique_keys(n, 61), wdgen.values(n, 62)
+    q = wdgen.interleaved_queries(n, 61)
+    cv, cf = oracle.expected_unique(q, n, 61, 62)
+    for qg in (-1, 16, 0, 1, 4, 32):
+        with wd.Table(capacity_for(n, 0.97), 1, G) as t:
+            assert t.get_option(wd.WD_OPT_QUERY_GROUP_SIZE) == -1
+            t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)
+            assert t.get_option(wd.WD_OPT_QUERY_GROUP_SIZE) == qg
+            gv, gf = gpu_roundtrip(t, keys, vals, q)
+            assert np.array_equal(gf, cf) and np.array_equal(gv, cv), qg
+            # auto at load 0.97: 16
+            assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == (16 if qg < 0 else qg or G)
+            # erase every third key (found flags), then query past the tombstones
+            er = keys[::3]
+            df = t.erase(to_dev(er))
+            assert np.all(df.cpu().numpy() == 1)
+            # the next insert (updates of the rest) runs with the table's |g|
+            upd = keys[1::3]
+            t.insert(to_dev(upd), to_dev(vals[1::3] ^ np.uint32(0x5A5A5A5A)))
+            assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == G
+            ov, of = t.retrieve(to_dev(keys))
+            gv, gf = from_dev(ov), of.cpu().numpy()
+            assert t.sync() == 0 and t.size() == n - er.size
+        want_f = np.ones(n, np.uint8); want_f[::3] = 0
+        want_v = vals.copy(); want_v[1::3] ^= np.uint32(0x5A5A5A5A)
+        assert np.array_equal(gf, want_f), qg
+        assert np.array_equal(gv[want_f == 1], want_v[want_f == 1]), qg
 
 
 @pytest.mark.parametrize("G,mode,flags", [(1, 1, 3), (4, 1, 3), (32, 1, 3), (2, 2, 3), (4, 2, 3),
@@ -153,6 +191,7 @@ def test_duplicates_upsert(wd, G, mode, flags):
     with wd.Table(capacity_for(150_000, 0.9), 1, G) as t:
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
+        t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
         t.insert(to_dev(keys), to_dev(vals))
         q = np.arange(160_000, dtype=np.uint32)
         ov, of = t.retrieve(to_dev(q))
@@ -284,6 +323,7 @@ def test_zipf_duplicates(wd, G, mode, flags):
     with wd.Table(capacity_for(distinct, 0.95), 1, G) as t:   # load = actual occupancy
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
+        t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
         q = np.concatenate([np.unique(keys), wdgen.unique_keys(1000, 99)])
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0
@@ -331,6 +371,7 @@ def test_scrambled_query_order(wd, G, V, n):
         with wd.Table(capacity_for(n, 0.95), 1, G) as t:
             t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
             t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
+            t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
             gv, gf = gpu_roundtrip(t, keys, vals, q)
             assert t.sync() == 0 and t.size() == n
         assert np.array_equal(gf, cf) and np.array_equal(gv, cv), flags
@@ -343,6 +384,7 @@ def test_window_split_parity(wd, G, V):
     q = wdgen.interleaved_queries(n, 33)
     with wd.Table(capacity_for(n, 0.97), 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
+        t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0 and t.size() == n
     cv, cf = oracle.expected_unique(q, n, 33, 34)
@@ -352,6 +394,7 @@ def test_window_split_parity(wd, G, V):
     dv = wdgen.values(200_000, 36)
     with wd.Table(capacity_for(60_000, 0.9), 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
+        t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
         qq = np.arange(61_000, dtype=np.uint32)
         gv, gf = gpu_roundtrip(t, dk, dv, qq)
         m = oracle.Map(200_000, dup_mode=True)
@@ -436,6 +479,7 @@ def test_span_read_ahead(wd, G, span):
     with wd.Table(capacity_for(n, 0.99), 1, G) as t:
         t.set_option(wd.WD_OPT_PROBE_MODE, 2)
         t.set_option(wd.WD_OPT_SPAN, span)
+        t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0 and t.size() == n
         df = t.erase(to_dev(q[: n // 2]))             # deletion runs the same probe

@@ -3,7 +3,8 @@
     python tools/rates.py LOG2N G [alpha] [key=value ...]
 
 keys: slices=<WD_OPT_SLICES>, v=<WD_OPT_SLOTS_PER_LANE>, k=<WD_OPT_KEYS_IN_FLIGHT>,
-span=<WD_OPT_SPAN>, reps=<timed repetitions>.  The kernel variant follows the environment
+span=<WD_OPT_SPAN>, reps=<timed repetitions>, qg=<|g| of the retrieve calls> (any |g| probes
+the same sequence; default the table's).  The kernel variant follows the environment
 (WD_PROBE_KERNEL=classic for the round-1 kernel).  Device-resident unique keys; every query
 checked against the closed form after the timed runs."""
 import json
@@ -28,6 +29,7 @@ def main():
     alpha = float(sys.argv[3]) if len(sys.argv) > 3 and "=" not in sys.argv[3] else 0.95
     kv = dict(a.split("=") for a in sys.argv[3:] if "=" in a)
     reps = int(kv.pop("reps", 5))
+    qg = int(kv.pop("qg", G))
     qmode = kv.pop("q", "")                 # inter: config 1 (all keys + as many absent,
     inter = qmode == "inter"                # interleaved); miss: absent keys only
     n = 1 << lg
@@ -44,9 +46,11 @@ def main():
         for r in range(reps + 1):
             a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
             t.clear(s)
+            t.set_option(wd.WD_OPT_GROUP_SIZE, G)
             a.record(s)
             t.insert(keys, vals, s)
             b.record(s)
+            t.set_option(wd.WD_OPT_GROUP_SIZE, qg)
             t.retrieve(qk, vo, fo, s)
             c.record(s)
             torch.cuda.synchronize()
@@ -57,7 +61,9 @@ def main():
         t.phase_times()
         t.set_option(wd.WD_OPT_PHASE_TIMING, 1)
         t.clear(s)
+        t.set_option(wd.WD_OPT_GROUP_SIZE, G)
         t.insert(keys, vals, s)
+        t.set_option(wd.WD_OPT_GROUP_SIZE, qg)
         ph_ins = {k: round(v[0], 4) for k, v in t.phase_times().items() if v[1]}
         t.retrieve(qk, vo, fo, s)
         ph_q = {k: round(v[0], 4) for k, v in t.phase_times().items() if v[1]}
@@ -65,7 +71,7 @@ def main():
         bad, first, found = gg.check_unique(qk, vo, fo, n, 11, 12)
         assert bad == 0 and found == (0 if qmode == "miss" else n)
         ims, qms = sum(ti) / len(ti), sum(tq) / len(tq)
-        print(json.dumps({"n_log2": lg, "G": G, "alpha": alpha, "opts": kv,
+        print(json.dumps({"n_log2": lg, "G": G, "query_G": qg, "alpha": alpha, "opts": kv,
                           "env": {k: v for k, v in os.environ.items() if k.startswith("WD_")},
                           "table_MB": t.capacity() * 8 / 1e6,
                           "insert_gops": n / ims / 1e6, "query_gops": nq / qms / 1e6, "queries": nq,
