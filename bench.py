@@ -847,30 +847,38 @@ def run_sweep(args, wd, gg, torch):
     for alpha in (0.8, 0.9, 0.95, 0.99):
         for G in (1, 2, 4, 8, 16, 32):
             with wd.Table(int(math.ceil(n / alpha)), 1, G) as t:
-                ti, tq, tauto = [], [], []
+                ti, tq, tauto, tiauto = [], [], [], []
                 for it in range(4):
-                    a, b, c, d = (torch.cuda.Event(enable_timing=True) for _ in range(4))
+                    a, b, c, d, e, f = (torch.cuda.Event(enable_timing=True) for _ in range(6))
+                    t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)    # the paper's: the table's |g|
+                    t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
                     t.clear(s)
                     a.record(s)
                     t.insert(keys, vals, s)
                     b.record(s)
-                    t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)     # the paper's: same |g|
                     t.retrieve(keys, vout, fout, s)
                     c.record(s)
-                    t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, -1)    # the library default (auto)
+                    t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, -1)    # the library defaults (auto)
+                    t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, -1)
                     t.retrieve(keys, vout, fout, s)
                     d.record(s)
+                    t.clear(s)
+                    e.record(s)
+                    t.insert(keys, vals, s)
+                    f.record(s)
                     torch.cuda.synchronize()
                     if it:
                         ti.append(a.elapsed_time(b))
                         tq.append(b.elapsed_time(c))
                         tauto.append(c.elapsed_time(d))
+                        tiauto.append(e.elapsed_time(f))
                 assert t.sync() == 0
                 pc = probe_cost(alpha, G)
                 ims, qms = sum(ti) / len(ti), sum(tq) / len(tq)
                 out.append({"sweep": "config2", "alpha": alpha, "G": G,
                             "insert_gops": n / ims / 1e6, "query_gops": n / qms / 1e6,
                             "query_gops_auto": n / (sum(tauto) / len(tauto)) / 1e6,
+                            "insert_gops_auto": n / (sum(tiauto) / len(tiauto)) / 1e6,
                             "insert_frac": n * (40 + 32 * pc["ins_sectors"]) / (ims * 1e-3) / 1e9 / hbm,
                             "query_frac": n * (9 + 32 * pc["hit_sectors"]) / (qms * 1e-3) / 1e9 / hbm})
     out += run_config1(wd, gg, torch)
@@ -917,7 +925,8 @@ def run_config1(wd, gg, torch):
     s = torch.cuda.current_stream()
     for G, qg in ((4, 0), (8, 0), (16, 0), (4, -1), (8, -1)):
         with wd.Table(int(math.ceil(n / 0.95)), 1, G) as t:
-            t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)   # 0: the paper's (queries with |g|)
+            t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)   # 0: the paper's (calls with |g|)
+            t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, qg)
             ti, tq = [], []
             for it in range(11):
                 a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))
@@ -1052,6 +1061,8 @@ def run_zipf(wd, gg, torch, log2n=27):
     for alpha in (0.8, 0.95):
         for G in (1, 2, 4, 8, 16):
             with wd.Table(int(math.ceil(distinct / alpha)), 1, G) as t:
+                t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)   # the paper's Fig. 8 grid: |g| as given
+                t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
                 ti, tq = [], []
                 for it in range(4):
                     a, b, c = (torch.cuda.Event(enable_timing=True) for _ in range(3))

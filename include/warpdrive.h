@@ -269,8 +269,16 @@ typedef enum {
                                 on B200 (profiles/r02/sweep_r02o.jsonl, query_group.jsonl;
                                 2^28 keys): alpha 0.95 hits on |g| = 1 / 2 / 4 / 32 tables
                                 7.0 / 10.4 / 17.6 / 19.0 -> 24.2 / 24.2 / 24.3 / 26.6 G/s,
-                                misses on |g| = 4 2.9 -> 7.9 G/s.  0: the inserts' |g| (the
+                                misses on |g| = 4 2.9 -> 7.9 G/s.  0: the table's |g| (the
                                 paper's setting); else 1..32. */
+    WD_OPT_INSERT_GROUP_SIZE = 17, /* |g| of wd_insert calls.  The slot an insert takes (the
+                                leftmost empty slot of its sequence, or its key's slot) is the
+                                same for any |g|, so the layout is too.  -1 (default):
+                                auto, 16 on A = 16 tables, 8 on A = 4 tables (tables created
+                                with |g| = 0 keep the choice by load).  Measured (2^28 keys,
+                                alpha 0.95): |g| 1 / 2 / 4 / 32 tables 9.7 / 14.4 / 20.7 / 15.9
+                                -> 22.1 / 22.1 / 22.1 / 23.5 G inserts/s.  0: the table's |g|
+                                (the paper's setting); else 1..32. */
     WD_OPT_N_SHARDS = 100,   /* read-only: m */
     WD_OPT_RANK = 101,       /* read-only: this process's rank (0 unless rank mode) */
     WD_OPT_LOCAL_SHARDS = 102, /* read-only: shards owned by this process */

@@ -35,6 +35,7 @@ WD_OPT_EXCHANGE = 12
 WD_OPT_PHASE_TIMING = 13
 WD_OPT_AUTO_REBUILD = 15
 WD_OPT_QUERY_GROUP_SIZE = 16
+WD_OPT_INSERT_GROUP_SIZE = 17
 PHASES = ["h2d", "group", "multisplit", "exchange", "probe", "reverse", "unpermute", "d2h",
           "probe_query"]
 EXCHANGE_FUSED, EXCHANGE_COPY, EXCHANGE_NCCL = 0, 1, 2

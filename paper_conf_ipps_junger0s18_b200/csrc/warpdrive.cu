@@ -1262,19 +1262,29 @@ wd_status_t classify_io(wd_table* t, bool insert, IO& io, int shard) {
 // step): |g| = 8 is fastest up to alpha 0.9, |g| = 16 from 0.95 on (and for misses at any
 // load).  The load used is the projected one after this call, from a host-side upper
 // estimate of the size (no synchronisation).
-// Queries and erases use WD_OPT_QUERY_GROUP_SIZE: the same results for any |g|.  Auto
-// (default): the layout, hence the query cost, depends only on the load and the region
-// alignment A, not on the |g| the keys were inserted with; measured on B200
-// (profiles/r02/sweep_r02o.jsonl, 2^28 keys, hits): A = 16 tables: |g| 16 (one line per
-// window) at every load; A = 4 tables: |g| 8 up to a load of 0.93 (alpha 0.8 / 0.9: 32.2 /
-// 28.0 G/s against 27.1 / 26.1 with 16-slot windows, which straddle two lines there), |g|
-// 16 above (0.95 / 0.99: 24.3 / 20.2 against 24.0 / 18.2); misses favour 16 at any load.
+// Calls probe with their own |g| (reading C24): P:89 gives every |g| the same probe sequence,
+// and an insert's slot — the leftmost empty slot of the sequence — does not depend on the
+// window size, so the layout, hence the cost of every call, depends only on the load and on
+// the region alignment A fixed at creation.  Auto (default), measured on B200
+// (profiles/r02/sweep_r02o.jsonl, 2^28 keys; the table's |g| rows are the paper's setting):
+//  * inserts: 16-slot windows on line-aligned tables (A = 16: |g| 32 tables 15.9 -> 23.5 G/s
+//    at alpha 0.95), 8-slot windows on A = 4 tables (|g| 1 / 2 / 4: 9.7 / 14.4 / 20.7 ->
+//    22.1 G/s); tables created with |g| = 0 keep the dynamic choice by load;
+//  * queries / erases: 16-slot windows on A = 16 tables and above a projected load of 0.93,
+//    else 8 (alpha 0.8 / 0.9 on A = 4: 32.2 / 28.0 G/s against 27.1 / 26.1 with 16-slot
+//    windows, which straddle two lines there; 0.95 / 0.99: 24.3 / 20.2 against 24.0 / 18.2;
+//    misses favour 16 at any load).
+// Option value 0 restores the paper's setting (the table's |g|), > 0 forces a |g|.
 void pick_group_size(wd_table* t, int op, uint64_t n) {
   const double cap = double(wd_capacity(t));
   const double est = double(t->est_size) + (op == OP_INSERT ? double(n) : 0.0);
   const bool high = est / cap > 0.93;
-  t->G_ins = t->G ? t->G : (high ? 16 : 8);
-  if (op == OP_INSERT || t->qg == 0) t->G_used = t->G_ins;
+  const int table_g = t->G ? t->G : (high ? 16 : 8);        // the paper's |g| (0: P:245 by load)
+  if (t->ig == 0 || (t->ig < 0 && t->G == 0)) t->G_ins = table_g;
+  else if (t->ig > 0) t->G_ins = t->ig;
+  else t->G_ins = t->align >= 16 ? 16 : 8;
+  if (op == OP_INSERT) t->G_used = t->G_ins;
+  else if (t->qg == 0) t->G_used = table_g;
   else if (t->qg > 0) t->G_used = t->qg;
   else t->G_used = (t->align >= 16 || high) ? 16 : 8;
   if (op == OP_INSERT) t->est_size = std::min<uint64_t>(t->est_size + n, wd_capacity(t));
@@ -1846,6 +1856,11 @@ wd_status_t wd_set_option(wd_table_t* t, wd_option_t opt, int64_t v) {
         return fail(WD_ERR_INVALID_ARG, "query group size %lld", (long long)v);
       t->qg = int(v);
       return WD_OK;
+    case WD_OPT_INSERT_GROUP_SIZE:
+      if (v != -1 && v != 0 && v != 1 && v != 2 && v != 4 && v != 8 && v != 16 && v != 32)
+        return fail(WD_ERR_INVALID_ARG, "insert group size %lld", (long long)v);
+      t->ig = int(v);
+      return WD_OK;
     case WD_OPT_P_MAX:
       if (v < 0 || v > (1 << 26)) return fail(WD_ERR_INVALID_ARG, "p_max %lld", (long long)v);
       t->pmax = int(v);
@@ -1913,6 +1928,7 @@ int64_t wd_get_option(wd_table_t* t, wd_option_t opt) {
     case WD_OPT_GROUP_SIZE: return t->G;
     case WD_OPT_GROUP_SIZE_USED: return t->G_used;
     case WD_OPT_QUERY_GROUP_SIZE: return t->qg;
+    case WD_OPT_INSERT_GROUP_SIZE: return t->ig;
     case WD_OPT_REGION_ALIGN: return t->align;
     case WD_OPT_P_MAX: return t->pmax;
     case WD_OPT_BATCH: return int64_t(t->batch);

@@ -141,7 +141,8 @@ struct wd_table {
   int G = 4;          // |g|, or 0 = dynamic by load
   int G_used = 4;     // |g| of the current / last call
   int G_ins = 4;      // |g| of the last insert (dynamic |g|: by load)
-  int qg = -1;        // |g| of query / erase calls (WD_OPT_QUERY_GROUP_SIZE; -1 auto, 0 G_ins)
+  int qg = -1;        // |g| of query / erase calls (WD_OPT_QUERY_GROUP_SIZE; -1 auto, 0 table's)
+  int ig = -1;        // |g| of insert calls (WD_OPT_INSERT_GROUP_SIZE; -1 auto, 0 table's)
   uint32_t align = 4; // A of reading C2': 16 for tables created with |g| >= 16, else 4
   uint64_t est_size = 0;   // host-side upper estimate of the stored keys (no sync needed)
   int pmax = 0;      // 0: p_max = nb (full period, C4'), else explicit

@@ -48,6 +48,7 @@ def test_erase_and_reinsert_parity(wd, G, V):
     with wd.Table(capacity_for(n, 0.8), 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)   # queries / erases with this |g| and V
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         t.insert(to_dev(keys), to_dev(vals))
         f = _erase(t, er)
         _check_found_once(f, er, set(keys.tolist()))
@@ -78,6 +79,8 @@ def test_erase_rebuild_serial_layout(wd, G, V):
     with wd.Table(4000, 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)   # queries / erases with this |g| and V
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         t.set_option(wd.WD_OPT_SERIAL, 1)
         t.insert(to_dev(keys), to_dev(vals))
         _erase(t, er)

@@ -31,6 +31,7 @@ def test_loopback_unique_parity(wd, m, G, mode):
     with wd.Table(capacity_for(n, 0.9), group_size=G, loopback_shards=m) as t:
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, -1 if mode == 0 else 0)   # 0: the table's |g|
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, -1 if mode == 0 else 0)
         t.set_option(wd.WD_OPT_BATCH, 9_000)  # many batches per shard: epochs wrap slots
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0, wd._lib.wd_last_error_message()

@@ -40,6 +40,7 @@ def test_config1_unique_parity(wd, G, mode, qg):
     with wd.Table(capacity_for(n, 0.95), 1, G) as t:
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)      # 0: queries with the table's |g|
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, qg)     # -1: the library's auto choice
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0
         assert t.size() == n
@@ -69,6 +70,7 @@ def test_alpha_and_keys_in_flight(wd, alpha, kif, mode):
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, kif)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0 and t.size() == n
     cv, cf = oracle.expected_unique(q, n, 7, 8)
@@ -90,6 +92,7 @@ def test_serial_layout_equals_fig3_replay(wd, G, mode):
     with wd.Table(3200, 1, G) as t:
         assert t.shard_capacity() == c
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         t.set_option(wd.WD_OPT_SERIAL, 1)
         t.insert(to_dev(keys), to_dev(vals))
         assert t.sync() == 0
@@ -111,7 +114,7 @@ def test_region_align_is_per_table(wd, Gc, Gi):
     r.insert(keys, vals)
     with wd.Table(2300, 1, Gc) as t:
         assert t.get_option(wd.WD_OPT_REGION_ALIGN) == A and t.capacity() == c
-        t.set_option(wd.WD_OPT_GROUP_SIZE, Gi)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, Gi)
         t.set_option(wd.WD_OPT_SERIAL, 1)
         t.insert(to_dev(keys), to_dev(vals))
         assert t.sync() == 0
@@ -134,6 +137,7 @@ def test_cross_group_size(wd, Gi, Gq, mi, mq):
     keys, vals = wdgen.unique_keys(n, 9), wdgen.values(n, 9)
     q = wdgen.interleaved_queries(n, 9)
     with wd.Table(capacity_for(n, 0.97), 1, Gi) as t:
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         t.set_option(wd.WD_OPT_PROBE_MODE, mi)
         t.insert(to_dev(keys), to_dev(vals))
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, Gq)
@@ -146,37 +150,58 @@ def test_cross_group_size(wd, Gi, Gq, mi, mq):
 
 @pytest.mark.parametrize("G", [1, 2, 4, 8, 16, 32])
 def test_query_group_size(wd, G):
-    # WD_OPT_QUERY_GROUP_SIZE (default -1 = auto): retrieve / erase with a |g| other than the
-    # inserts' — P:89, every result is the same: hits, misses (long chains at alpha 0.97),
-    # erase flags, queries past tombstones, and the values of updated keys
+    # WD_OPT_QUERY_GROUP_SIZE / WD_OPT_INSERT_GROUP_SIZE (default -1 = auto): calls probe with
+    # a |g| other than the table's — P:89, every result is the same: hits, misses (long
+    # chains at alpha 0.97), erase flags, queries past tombstones, updates of existing keys
     n = 120_001
     keys, vals = wdgen.unique_keys(n, 61), wdgen.values(n, 62)
     q = wdgen.interleaved_queries(n, 61)
     cv, cf = oracle.expected_unique(q, n, 61, 62)
-    for qg in (-1, 16, 0, 1, 4, 32):
+    auto_ins = 16 if G >= 16 else 8                       # by region alignment A
+    for qg, ig in ((-1, -1), (16, 0), (0, 0), (1, -1), (4, 0), (32, 32), (-1, 1)):
         with wd.Table(capacity_for(n, 0.97), 1, G) as t:
             assert t.get_option(wd.WD_OPT_QUERY_GROUP_SIZE) == -1
+            assert t.get_option(wd.WD_OPT_INSERT_GROUP_SIZE) == -1
             t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, qg)
+            t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, ig)
             assert t.get_option(wd.WD_OPT_QUERY_GROUP_SIZE) == qg
             gv, gf = gpu_roundtrip(t, keys, vals, q)
-            assert np.array_equal(gf, cf) and np.array_equal(gv, cv), qg
+            assert np.array_equal(gf, cf) and np.array_equal(gv, cv), (qg, ig)
             # auto at load 0.97: 16
             assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == (16 if qg < 0 else qg or G)
             # erase every third key (found flags), then query past the tombstones
             er = keys[::3]
             df = t.erase(to_dev(er))
             assert np.all(df.cpu().numpy() == 1)
-            # the next insert (updates of the rest) runs with the table's |g|
-            upd = keys[1::3]
+            upd = keys[1::3]                              # updates of existing keys
             t.insert(to_dev(upd), to_dev(vals[1::3] ^ np.uint32(0x5A5A5A5A)))
-            assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == G
+            assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == (auto_ins if ig < 0 else ig or G)
             ov, of = t.retrieve(to_dev(keys))
             gv, gf = from_dev(ov), of.cpu().numpy()
             assert t.sync() == 0 and t.size() == n - er.size
         want_f = np.ones(n, np.uint8); want_f[::3] = 0
         want_v = vals.copy(); want_v[1::3] ^= np.uint32(0x5A5A5A5A)
-        assert np.array_equal(gf, want_f), qg
-        assert np.array_equal(gv[want_f == 1], want_v[want_f == 1]), qg
+        assert np.array_equal(gf, want_f), (qg, ig)
+        assert np.array_equal(gv[want_f == 1], want_v[want_f == 1]), (qg, ig)
+
+
+def test_auto_insert_serial_layout(wd):
+    # the auto insert |g| (8 on A = 4 tables, 16 on A = 16) lays the keys out exactly as the
+    # paper's |g| does: serial layout = the Fig. 3 replay with the table's |g| and geometry
+    n = 2500
+    for G in (1, 2, 4, 32):
+        A = oracle.region_align_for(G)
+        c = oracle.physical_capacity(2700, A)
+        keys = np.concatenate([wdgen.unique_keys(n, 71), wdgen.unique_keys(100, 71)])
+        vals = wdgen.values(n + 100, 72)
+        r = oracle.Replay(c, G, align=A)
+        r.insert(keys, vals)
+        with wd.Table(2700, 1, G) as t:
+            t.set_option(wd.WD_OPT_SERIAL, 1)
+            t.insert(to_dev(keys), to_dev(vals))
+            assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == (16 if G >= 16 else 8)
+            assert t.sync() == 0
+            assert np.array_equal(t.dump(), r.table), G
 
 
 @pytest.mark.parametrize("G,mode,flags", [(1, 1, 3), (4, 1, 3), (32, 1, 3), (2, 2, 3), (4, 2, 3),
@@ -192,6 +217,7 @@ def test_duplicates_upsert(wd, G, mode, flags):
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         t.insert(to_dev(keys), to_dev(vals))
         q = np.arange(160_000, dtype=np.uint32)
         ov, of = t.retrieve(to_dev(q))
@@ -324,6 +350,7 @@ def test_zipf_duplicates(wd, G, mode, flags):
         t.set_option(wd.WD_OPT_PROBE_MODE, mode)
         t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         q = np.concatenate([np.unique(keys), wdgen.unique_keys(1000, 99)])
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0
@@ -351,6 +378,7 @@ def test_window_split_serial_layout(wd, G, V):
     r.insert(keys, vals)
     with wd.Table(2700, 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         t.set_option(wd.WD_OPT_SERIAL, 1)
         t.insert(to_dev(keys), to_dev(vals))
         assert t.sync() == 0
@@ -372,6 +400,7 @@ def test_scrambled_query_order(wd, G, V, n):
             t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
             t.set_option(wd.WD_OPT_KERNEL_FLAGS, flags)
             t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
+            t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
             gv, gf = gpu_roundtrip(t, keys, vals, q)
             assert t.sync() == 0 and t.size() == n
         assert np.array_equal(gf, cf) and np.array_equal(gv, cv), flags
@@ -385,6 +414,7 @@ def test_window_split_parity(wd, G, V):
     with wd.Table(capacity_for(n, 0.97), 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0 and t.size() == n
     cv, cf = oracle.expected_unique(q, n, 33, 34)
@@ -395,6 +425,7 @@ def test_window_split_parity(wd, G, V):
     with wd.Table(capacity_for(60_000, 0.9), 1, G) as t:
         t.set_option(wd.WD_OPT_SLOTS_PER_LANE, V)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         qq = np.arange(61_000, dtype=np.uint32)
         gv, gf = gpu_roundtrip(t, dk, dv, qq)
         m = oracle.Map(200_000, dup_mode=True)
@@ -469,6 +500,7 @@ def test_span_read_ahead(wd, G, span):
         t.set_option(wd.WD_OPT_PROBE_MODE, 2)          # one lane per window (V = |g|)
         t.set_option(wd.WD_OPT_SPAN, span)
         assert t.get_option(wd.WD_OPT_SPAN) == span
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         t.set_option(wd.WD_OPT_SERIAL, 1)
         t.insert(to_dev(keys), to_dev(vals))
         assert t.sync() == 0
@@ -480,6 +512,7 @@ def test_span_read_ahead(wd, G, span):
         t.set_option(wd.WD_OPT_PROBE_MODE, 2)
         t.set_option(wd.WD_OPT_SPAN, span)
         t.set_option(wd.WD_OPT_QUERY_GROUP_SIZE, 0)
+        t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, 0)
         gv, gf = gpu_roundtrip(t, keys, vals, q)
         assert t.sync() == 0 and t.size() == n
         df = t.erase(to_dev(q[: n // 2]))             # deletion runs the same probe
