@@ -565,6 +565,51 @@ def test_slice_grouped_insert(wd, G, slices):
         assert np.array_equal(from_dev(ov), v2)
 
 
+def _fmix32_inv(h: np.ndarray) -> np.ndarray:
+    """inverse of MurmurHash3's fmix32 (test helper: keys with chosen first-region slices)"""
+    x = h.astype(np.uint64)
+    m = np.uint64(0xFFFFFFFF)
+    x ^= x >> np.uint64(16)
+    x = (x * np.uint64(pow(0xC2B2AE35, -1, 1 << 32))) & m
+    x ^= (x >> np.uint64(13)) ^ (x >> np.uint64(26))
+    x = (x * np.uint64(pow(0x85EBCA6B, -1, 1 << 32))) & m
+    x ^= x >> np.uint64(16)
+    return x.astype(np.uint32)
+
+
+@pytest.mark.parametrize("skew", ["one_slice", "ninety_percent", "last_slice_and_ragged"])
+def test_slice_grouped_insert_skewed(wd, skew):
+    # the segment-mode multisplit with skewed slice counts: every key's first region in one
+    # slice (all blocks' counts in one destination), 90 % in one slice, or all in the last
+    # slice with a ragged tail; keys built through the inverse of fmix32 (slice = top 5 bits
+    # of fmix32(k + seed), seed 0 on a fresh table)
+    rng = np.random.default_rng(5)
+    n = (1 << 20) + 77
+    top = {"one_slice": 0, "ninety_percent": 5, "last_slice_and_ragged": 31}[skew]
+    h = rng.choice(1 << 27, size=n, replace=False).astype(np.uint64) + (np.uint64(top) << np.uint64(27))
+    if skew == "ninety_percent":
+        k = n // 10
+        h[:k] = rng.choice(1 << 32, size=k, replace=False).astype(np.uint64)
+        h = np.unique(h)
+        n = h.size
+    keys = _fmix32_inv(h.astype(np.uint32))
+    assert np.array_equal(oracle.fmix32_many(keys), h.astype(np.uint32))   # the inverse, pinned
+    keep = keys != np.uint32(0xFFFFFFFF)
+    keys = keys[keep]
+    n = keys.size
+    vals = wdgen.values(n, 81)
+    absent = wdgen.unique_keys(50_000, 82)
+    absent = absent[~np.isin(absent, keys)]
+    with wd.Table(capacity_for(n, 0.6), 1, 16) as t:
+        t.set_option(wd.WD_OPT_SLICES, 32)
+        t.insert(to_dev(keys), to_dev(vals))
+        assert t.sync() == 0 and t.size() == n
+        ov, of = t.retrieve(to_dev(np.concatenate([keys, absent])))
+        gv, gf = from_dev(ov), of.cpu().numpy()
+    assert np.all(gf[:n] == 1) and np.array_equal(gv[:n], vals)
+    assert np.all(gf[n:] == 0)
+
+
 def test_slice_grouped_insert_chunks(wd):
     # more than one 2^26-pair chunk (auto slices on an HBM-sized table), ragged tail;
     # every query checked against the closed form on a sample
