@@ -934,7 +934,7 @@ wd_status_t cascade_op(wd_table* t, int op, std::vector<IO>& ios, cudaStream_t s
                                         : wd::multisplit_kernel<true, 1, false, false, 0>)
                        : (t->pmode == 1 ? wd::multisplit_kernel<false, 1, false, false, 1>
                                         : wd::multisplit_kernel<false, 1, false, false, 0>);
-    const uint64_t tiles = (cnt + wd::kMs2Tile - 1) / wd::kMs2Tile;
+    const uint64_t tiles = (cnt + wd::kMs2TileC - 1) / wd::kMs2TileC;
     const int grid = int(std::min<uint64_t>(tiles, uint64_t(t->sm_count) * blocks_per_sm(kern)));
     kern<<<grid, wd::kBlock, 0, s.s_main>>>(dk, insert ? dv : nullptr, cnt, dst, s.cursor[slot], nullptr, 0,
                                              insert ? nullptr : s.pos[slot], m, t->pseed, B, s.counters);

@@ -4,7 +4,7 @@
 // (read 4 + 4 B, write 8 B per pair) as the streaming speed of light.  Every output is
 // checked on the host: each slice's range holds only keys of that slice, and the values
 // (= input indices) form a permutation.
-// Build (compile-time variants via -DWD_MS2_IPT=.. -DWD_MS2_MINB=..):
+// Build (compile-time variants via -DWD_MS2_IPT=.. -DWD_MS2_MINB=.., cursor mode -DWD_MS2_IPTC/MINBC):
 //   nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -Iinclude \
 //        -o tools/ms_bench tools/ms_bench.cu
 // Run: tools/ms_bench [log2 n = 28] [reps = 10]
@@ -142,7 +142,7 @@ int main(int argc, char** argv) {
     for (int d = 0; d < m; ++d) dd.p[d] = rbuf + d * B;
     auto run2 = [&](bool pairs) {
       CK(cudaMemsetAsync(cursor, 0, m * 8));
-      const int g = std::min<uint64_t>((nc + wd::kMs2Tile - 1) / wd::kMs2Tile,
+      const int g = std::min<uint64_t>((nc + wd::kMs2TileC - 1) / wd::kMs2TileC,
                                        uint64_t(sms) * occ(wd::multisplit_kernel<true, 1, false, false, 0>));
       if (pairs) wd::multisplit_kernel<true, 1, false, false, 0><<<g, wd::kBlock>>>(k + mis, v + mis, nc, dd, cursor, nullptr, 0, nullptr, m, seed, B, ctr);
       else wd::multisplit_kernel<false, 1, false, false, 0><<<g, wd::kBlock>>>(k + mis, nullptr, nc, dd, cursor, nullptr, 0, posb, m, seed, B, ctr);
@@ -178,12 +178,13 @@ int main(int argc, char** argv) {
       }
       if (tot != nc) ++bad;
       ok &= bad == 0;
-      printf("{\"cascade_m\": %d, \"n\": %llu, \"misaligned\": %d, \"pairs\": %d, \"ms\": %.4f, \"bad\": %llu}\n", m,
-             (unsigned long long)nc, mis, int(pairs), b, (unsigned long long)bad);
+      printf("{\"cascade_m\": %d, \"n\": %llu, \"misaligned\": %d, \"pairs\": %d, \"ms\": %.4f, \"ipt\": %d, \"bad\": %llu}\n", m,
+             (unsigned long long)nc, mis, int(pairs), b, WD_MS2_IPTC, (unsigned long long)bad);
     }
     CK(cudaFree(rbuf)); CK(cudaFree(posb));
   };
   cascade(n, 8, true);
+  cascade(n / 2, 2, true);   // pos offsets hold 27 bits: batches of <= 2^27 items per owner
   for (int mis : {0, 1})
     for (int mm : {2, 3})
       for (uint64_t nc : {1ull, 100ull, 3656ull, 4096ull, 8192ull, 9000ull, 60000ull, 1000003ull}) cascade(nc, mm, false, mis);
