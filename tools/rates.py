@@ -3,7 +3,7 @@
     python tools/rates.py LOG2N G [alpha] [key=value ...]
 
 keys: slices=<WD_OPT_SLICES>, v=<WD_OPT_SLOTS_PER_LANE>, k=<WD_OPT_KEYS_IN_FLIGHT>,
-span=<WD_OPT_SPAN>, reps=<timed repetitions>, qg=<|g| of the retrieve calls> (any |g| probes
+span=<WD_OPT_SPAN>, ig=<WD_OPT_INSERT_GROUP_SIZE>, reps=<timed repetitions>, qg=<|g| of the retrieve calls> (any |g| probes
 the same sequence; default the table's).  The kernel variant follows the environment
 (WD_PROBE_KERNEL=classic for the round-1 kernel).  Device-resident unique keys; every query
 checked against the closed form after the timed runs."""
@@ -20,6 +20,7 @@ import paper_conf_ipps_junger0s18_b200 as wd  # noqa: E402
 import wdgen.gpu as gg  # noqa: E402
 
 OPT = {"slices": wd.WD_OPT_SLICES, "v": wd.WD_OPT_SLOTS_PER_LANE, "k": wd.WD_OPT_KEYS_IN_FLIGHT,
+       "ig": wd.WD_OPT_INSERT_GROUP_SIZE,
        "span": wd.WD_OPT_SPAN, "mode": wd.WD_OPT_PROBE_MODE,
        "flags": wd.WD_OPT_KERNEL_FLAGS}
 
