@@ -274,8 +274,8 @@ typedef enum {
     WD_OPT_INSERT_GROUP_SIZE = 17, /* |g| of wd_insert calls.  The slot an insert takes (the
                                 leftmost empty slot of its sequence, or its key's slot) is the
                                 same for any |g|, so the layout is too.  -1 (default):
-                                auto, 16 on A = 16 tables, 8 on A = 4 tables (tables created
-                                with |g| = 0 keep the choice by load).  Measured (2^28 keys,
+                                auto, 16 on A = 16 tables and on shards of <= 64 MB, else 8
+                                (tables created with |g| = 0 keep the choice by load).  Measured (2^28 keys,
                                 alpha 0.95): |g| 1 / 2 / 4 / 32 tables 9.7 / 14.4 / 20.7 / 15.9
                                 -> 22.1 / 22.1 / 22.1 / 23.5 G inserts/s.  0: the table's |g|
                                 (the paper's setting); else 1..32. */

@@ -1268,8 +1268,11 @@ wd_status_t classify_io(wd_table* t, bool insert, IO& io, int shard) {
 // the region alignment A fixed at creation.  Auto (default), measured on B200
 // (profiles/r02/sweep_r02o.jsonl, 2^28 keys; the table's |g| rows are the paper's setting):
 //  * inserts: 16-slot windows on line-aligned tables (A = 16: |g| 32 tables 15.9 -> 23.5 G/s
-//    at alpha 0.95), 8-slot windows on A = 4 tables (|g| 1 / 2 / 4: 9.7 / 14.4 / 20.7 ->
-//    22.1 G/s); tables created with |g| = 0 keep the dynamic choice by load;
+//    at alpha 0.95) and on shards of <= 64 MB (L2-resident: 2^20 / 2^22 keys 6.9 / 19.8 ->
+//    11.0 / 23.9 G/s against 8-slot windows), 8-slot windows on larger A = 4 tables (|g| 1 /
+//    2 / 4: 9.7 / 14.4 / 20.7 -> 22.1 G/s; 16-slot windows there: 15.4, they straddle two
+//    lines; profiles/r02/insert_group.jsonl); tables created with |g| = 0 keep the dynamic
+//    choice by load;
 //  * queries / erases: 16-slot windows on A = 16 tables and above a projected load of 0.93,
 //    else 8 (alpha 0.8 / 0.9 on A = 4: 32.2 / 28.0 G/s against 27.1 / 26.1 with 16-slot
 //    windows, which straddle two lines there; 0.95 / 0.99: 24.3 / 20.2 against 24.0 / 18.2;
@@ -1282,7 +1285,7 @@ void pick_group_size(wd_table* t, int op, uint64_t n) {
   const int table_g = t->G ? t->G : (high ? 16 : 8);        // the paper's |g| (0: P:245 by load)
   if (t->ig == 0 || (t->ig < 0 && t->G == 0)) t->G_ins = table_g;
   else if (t->ig > 0) t->G_ins = t->ig;
-  else t->G_ins = t->align >= 16 ? 16 : 8;
+  else t->G_ins = (t->align >= 16 || t->local[0].cap * 8 <= (64ull << 20)) ? 16 : 8;
   if (op == OP_INSERT) t->G_used = t->G_ins;
   else if (t->qg == 0) t->G_used = table_g;
   else if (t->qg > 0) t->G_used = t->qg;

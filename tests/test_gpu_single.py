@@ -157,7 +157,7 @@ def test_query_group_size(wd, G):
     keys, vals = wdgen.unique_keys(n, 61), wdgen.values(n, 62)
     q = wdgen.interleaved_queries(n, 61)
     cv, cf = oracle.expected_unique(q, n, 61, 62)
-    auto_ins = 16 if G >= 16 else 8                       # by region alignment A
+    auto_ins = 16                                         # A = 16, or a shard <= 64 MB
     for qg, ig in ((-1, -1), (16, 0), (0, 0), (1, -1), (4, 0), (32, 32), (-1, 1)):
         with wd.Table(capacity_for(n, 0.97), 1, G) as t:
             assert t.get_option(wd.WD_OPT_QUERY_GROUP_SIZE) == -1
@@ -186,22 +186,24 @@ def test_query_group_size(wd, G):
 
 
 def test_auto_insert_serial_layout(wd):
-    # the auto insert |g| (8 on A = 4 tables, 16 on A = 16) lays the keys out exactly as the
-    # paper's |g| does: serial layout = the Fig. 3 replay with the table's |g| and geometry
+    # the auto insert |g| (16 on small shards and A = 16 tables, 8 on A = 4 shards > 64 MB)
+    # lays the keys out exactly as the paper's |g| does: serial layout = the Fig. 3 replay
+    # with the table's |g| and geometry
     n = 2500
-    for G in (1, 2, 4, 32):
+    for G, cap, want in ((1, 2700, 16), (2, 2700, 16), (4, 2700, 16), (32, 2700, 16),
+                         (4, 9_000_000, 8), (16, 9_000_000, 16)):
         A = oracle.region_align_for(G)
-        c = oracle.physical_capacity(2700, A)
+        c = oracle.physical_capacity(cap, A)
         keys = np.concatenate([wdgen.unique_keys(n, 71), wdgen.unique_keys(100, 71)])
         vals = wdgen.values(n + 100, 72)
         r = oracle.Replay(c, G, align=A)
         r.insert(keys, vals)
-        with wd.Table(2700, 1, G) as t:
+        with wd.Table(cap, 1, G) as t:
             t.set_option(wd.WD_OPT_SERIAL, 1)
             t.insert(to_dev(keys), to_dev(vals))
-            assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == (16 if G >= 16 else 8)
+            assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == want, (G, cap)
             assert t.sync() == 0
-            assert np.array_equal(t.dump(), r.table), G
+            assert np.array_equal(t.dump(), r.table), (G, cap)
 
 
 @pytest.mark.parametrize("G,mode,flags", [(1, 1, 3), (4, 1, 3), (32, 1, 3), (2, 2, 3), (4, 2, 3),
