@@ -74,6 +74,8 @@ typedef enum {
  * destroyed (environment WD_L2_FETCH_BYTES=<bytes> overrides, 0 = leave it alone).
  * n_gpus > 1: one shard per device 0..n_gpus-1, keys owned by shard p(k),
  * peer access over NVLink; host input is split into n_gpus contiguous chunks.
+ * (Test hook: with environment WD_MULTI_SAME_DEVICE set, all shards live on the current
+ * device, so this mode's code runs on a one-GPU box; n_gpus may then exceed the count.)
  * capacity: total slots c (alpha = n / c).  Each shard gets ceil(c / m) slots,
  * rounded up to a multiple of A and to at least 32 (the 32-slot region, Fig. 3 Line 6), then
  * until the region count is prime (C13').  A = the region-start alignment (C2'):

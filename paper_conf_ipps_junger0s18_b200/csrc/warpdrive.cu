@@ -1519,7 +1519,11 @@ wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size) {
     fail(WD_ERR_CUDA, "no CUDA device");
     return nullptr;
   }
-  if (n_gpus < 1 || n_gpus > ndev) {
+  // test hook (tests/test_gpu_multi_samedev.py): every shard of a multi-GPU table on the
+  // current device, so the single-process multi-GPU code (per-device streams, host-input
+  // split, _sharded calls, device-pointer rules) runs on a one-GPU box
+  const bool same_dev = getenv("WD_MULTI_SAME_DEVICE") != nullptr;
+  if (n_gpus < 1 || (n_gpus > ndev && !same_dev)) {
     fail(WD_ERR_INVALID_ARG, "n_gpus %d not in [1, %d visible]", n_gpus, ndev);
     return nullptr;
   }
@@ -1527,12 +1531,12 @@ wd_table_t* wd_create(uint64_t capacity, int n_gpus, int group_size) {
   if (!t) return nullptr;
   int cur = 0;
   cudaGetDevice(&cur);
-  cudaDeviceGetAttribute(&t->sm_count, cudaDevAttrMultiProcessorCount, n_gpus == 1 ? cur : 0);
+  cudaDeviceGetAttribute(&t->sm_count, cudaDevAttrMultiProcessorCount, n_gpus == 1 || same_dev ? cur : 0);
   const uint64_t c = shard_cap(capacity, n_gpus, t->align);
   t->local.resize(n_gpus);
   for (int d = 0; d < n_gpus; ++d) {
-    const int dev = n_gpus == 1 ? cur : d;
-    if (n_gpus > 1) {
+    const int dev = n_gpus == 1 || same_dev ? cur : d;
+    if (n_gpus > 1 && !same_dev) {
       DeviceGuard g(dev);
       for (int p = 0; p < n_gpus; ++p)
         if (p != dev) {
