@@ -277,6 +277,7 @@ typedef enum {
                                 leftmost empty slot of its sequence, or its key's slot) is the
                                 same for any |g|, so the layout is too.  -1 (default):
                                 auto, 16 on A = 16 tables and on shards of <= 64 MB, else 8
+                                up to 24 GB shards and the table's |g| (at least 4) above
                                 (tables created with |g| = 0 keep the choice by load).  Measured (2^28 keys,
                                 alpha 0.95): |g| 1 / 2 / 4 / 32 tables 9.7 / 14.4 / 20.7 / 15.9
                                 -> 22.1 / 22.1 / 22.1 / 23.5 G inserts/s.  0: the table's |g|

@@ -1271,8 +1271,11 @@ wd_status_t classify_io(wd_table* t, bool insert, IO& io, int shard) {
 //    at alpha 0.95) and on shards of <= 64 MB (L2-resident: 2^20 / 2^22 keys 6.9 / 19.8 ->
 //    11.0 / 23.9 G/s against 8-slot windows), 8-slot windows on larger A = 4 tables (|g| 1 /
 //    2 / 4: 9.7 / 14.4 / 20.7 -> 22.1 G/s; 16-slot windows there: 15.4, they straddle two
-//    lines; profiles/r02/insert_group.jsonl); tables created with |g| = 0 keep the dynamic
-//    choice by load;
+//    lines; profiles/r02/insert_group.jsonl) up to 24 GB shards (2^29 / 2^30 / 2^31 keys at
+//    |g| 4: 20.7 / 20.2 / 19.0 -> 22.0 / 20.8 / 20.0 G/s); above, where a slice no longer
+//    fits the L2 (config 3's 36 GB: 282 MB slices), the table's |g|, at least 4 (|g| 4:
+//    21.9 against 20.0 G/s with 8-slot windows; profiles/r02/insert_group_large.jsonl);
+//    tables created with |g| = 0 keep the dynamic choice by load;
 //  * queries / erases: 16-slot windows on A = 16 tables and above a projected load of 0.93,
 //    else 8 (alpha 0.8 / 0.9 on A = 4: 32.2 / 28.0 G/s against 27.1 / 26.1 with 16-slot
 //    windows, which straddle two lines there; 0.95 / 0.99: 24.3 / 20.2 against 24.0 / 18.2;
@@ -1285,7 +1288,8 @@ void pick_group_size(wd_table* t, int op, uint64_t n) {
   const int table_g = t->G ? t->G : (high ? 16 : 8);        // the paper's |g| (0: P:245 by load)
   if (t->ig == 0 || (t->ig < 0 && t->G == 0)) t->G_ins = table_g;
   else if (t->ig > 0) t->G_ins = t->ig;
-  else t->G_ins = (t->align >= 16 || t->local[0].cap * 8 <= (64ull << 20)) ? 16 : 8;
+  else if (t->align >= 16 || t->local[0].cap * 8 <= (64ull << 20)) t->G_ins = 16;
+  else t->G_ins = double(t->local[0].cap) * 8 > 24e9 ? std::max(t->G, 4) : 8;
   if (op == OP_INSERT) t->G_used = t->G_ins;
   else if (t->qg == 0) t->G_used = table_g;
   else if (t->qg > 0) t->G_used = t->qg;

@@ -206,6 +206,22 @@ def test_auto_insert_serial_layout(wd):
             assert np.array_equal(t.dump(), r.table), (G, cap)
 
 
+def test_auto_insert_group_large_table(wd):
+    # shards > 24 GB with A = 4 keep the table's |g| for inserts (config 3's regime); the map
+    # stays exact
+    n = 200_000
+    keys, vals = wdgen.unique_keys(n, 73), wdgen.values(n, 74)
+    q = wdgen.interleaved_queries(n, 73)
+    with wd.Table(3_300_000_000, 1, 4) as t:           # 26.4 GB
+        t.insert(to_dev(keys), to_dev(vals))
+        assert t.get_option(wd.WD_OPT_GROUP_SIZE_USED) == 4
+        ov, of = t.retrieve(to_dev(q))
+        gv, gf = from_dev(ov), of.cpu().numpy()
+        assert t.sync() == 0 and t.size() == n
+    cv, cf = oracle.expected_unique(q, n, 73, 74)
+    assert np.array_equal(gf, cf) and np.array_equal(gv, cv)
+
+
 @pytest.mark.parametrize("G,mode,flags", [(1, 1, 3), (4, 1, 3), (32, 1, 3), (2, 2, 3), (4, 2, 3),
                                           (8, 2, 3), (4, 0, 3), (4, 1, 0), (4, 2, 0), (1, 1, 1),
                                           (1, 1, 11), (4, 1, 11), (8, 0, 11), (8, 2, 8)])
