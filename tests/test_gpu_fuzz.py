@@ -1,7 +1,7 @@
 """Seeded randomized parity through the C-ABI: random sizes (ragged, tiny, empty), loads,
 table |g|, per-call insert / query |g| (reading C24), slice grouping, probe modes, keys in
 flight, duplicate fractions, the reserved key, erase and re-insert, host or device buffers,
-and loopback shards.  Every case replays its calls on the oracle's map (P:31 exact map,
+loopback shards, exchange modes and batch sizes.  Every case replays its calls on the oracle's map (P:31 exact map,
 P:185 upsert, P:91 delete) and compares every query: found flags exactly, values exactly for
 keys inserted once per call and v in V(k) for keys a call inserted several times."""
 import numpy as np
@@ -40,6 +40,8 @@ def _case(seed):
         "erase": float(r.choice([0.0, 0.25])),
         "host": bool(r.random() < 0.3),
         "shards": int(r.choice([1, 1, 1, 2, 3])),
+        "exchange": int(r.choice([0, 1])),   # fused peer stores / copy engine (cascade only)
+        "batch": int(r.choice([0, 5000, 1 << 16])),
     }
     if c["shards"] > 1:
         c["slices"] = 0                      # the cascade has no slice grouping
@@ -72,7 +74,7 @@ def test_fuzz_parity(wd, seed):
     # reused (reading C9'), so every re-inserted key takes a new slot (<= half of the erased
     # keys + 100 absent ones)
     cap = capacity_for(int(distinct * (1 + c["erase"] / 2)) + 150, c["alpha"]) + 64
-    kw = {"loopback_shards": c["shards"]} if c["shards"] > 1 else {}
+    kw = {"loopback_shards": c["shards"], "exchange": c["exchange"]} if c["shards"] > 1 else {}
     m = oracle.Map(max(n, 1) * 2, dup_mode=True)
     with (wd.Table(cap, group_size=c["G"], **kw) if kw else wd.Table(cap, 1, c["G"])) as t:
         t.set_option(wd.WD_OPT_INSERT_GROUP_SIZE, c["ig"])
@@ -82,6 +84,8 @@ def test_fuzz_parity(wd, seed):
         t.set_option(wd.WD_OPT_PROBE_MODE, c["mode"])
         if c["kif"]:
             t.set_option(wd.WD_OPT_KEYS_IN_FLIGHT, c["kif"])
+        if c["batch"]:
+            t.set_option(wd.WD_OPT_BATCH, c["batch"])        # pipeline / cascade batches
         if n:
             t.insert(_as_input(keys, c["host"]), _as_input(vals, c["host"]))
         m.insert(keys, vals)
