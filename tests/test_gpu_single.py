@@ -158,6 +158,12 @@ def test_query_group_size(wd, G):
     q = wdgen.interleaved_queries(n, 61)
     cv, cf = oracle.expected_unique(q, n, 61, 62)
     auto_ins = 16                                         # A = 16, or a shard <= 64 MB
+    with wd.Table(1000, 1, G) as t:                       # invalid values are refused
+        for opt in (wd.WD_OPT_QUERY_GROUP_SIZE, wd.WD_OPT_INSERT_GROUP_SIZE):
+            for bad in (-2, 3, 64):
+                with pytest.raises(Exception):
+                    t.set_option(opt, bad)
+            assert t.get_option(opt) == -1
     for qg, ig in ((-1, -1), (16, 0), (0, 0), (1, -1), (4, 0), (32, 32), (-1, 1)):
         with wd.Table(capacity_for(n, 0.97), 1, G) as t:
             assert t.get_option(wd.WD_OPT_QUERY_GROUP_SIZE) == -1
